@@ -1,0 +1,201 @@
+/*
+ * msp.h -- C ABI of libmsp, the B200 (sm_100a) merge-path sparse library.
+ *
+ * Implements the data-parallel hot path of S. Dalton, S. Baxter, D. Merrill,
+ * L. Olson, M. Garland, "Optimizing Sparse Matrix Operations on GPUs using
+ * Merge Path", IPDPS 2015 (PAPER.md, cited as P:<line>):
+ *
+ *   SpMV    y = A x        merge-path partition + segmented reduction with
+ *                          carry-out fix-up (Section III-A)
+ *   SpAdd   C = A + B      balanced-path set union of (row,col) tuples in
+ *                          two phases, count then fill (III-B)
+ *   SpGEMM  C = A B        expand / sort / compress with products balanced
+ *                          across CTAs by a search over the prefix sum S of
+ *                          the referenced B row lengths (III-C)
+ *
+ * Every entry point is extern "C", takes plain pointers and sizes, and never
+ * exposes a C++ or torch type.  DESIGN.md describes the kernels behind it.
+ *
+ * Conventions shared by all calls
+ * -------------------------------
+ * Matrices are CSR: row_offsets int32[nrows+1] with
+ * row_offsets[0] == 0 and row_offsets[nrows] == nnz, col_idx int32[nnz],
+ * vals float32 or float64 [nnz].  All array pointers in msp_csr and all
+ * vector / output / workspace pointers are DEVICE pointers unless the name
+ * ends in _host.  SpAdd and SpGEMM require each row's columns to be sorted
+ * ascending and unique (the input contract the method relies on);
+ * SpMV accepts any column order.  Indices are int32; product counts (Nprods)
+ * are int64 internally.
+ *
+ * Ownership: the caller allocates and owns every device buffer (inputs,
+ * outputs, workspaces).  The library never calls cudaMalloc/cudaFree and
+ * keeps no pointer after a call returns, except that the workspaces named in
+ * the *_numeric calls must be the ones the matching *_symbolic (or *_setup)
+ * call used, left untouched in between.  Workspaces must be zero-filled once
+ * before their first use (kernels leave their counters zeroed on exit).
+ *
+ * Streams: `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ * stream).  Calls marked "async" only enqueue work; calls that return a
+ * *_host scalar synchronise that stream before returning.
+ *
+ * Errors: every call returns an msp_status and never aborts.  Argument,
+ * shape and dtype checks run on the host before any launch.  Launch errors
+ * are returned as MSP_ERR_CUDA with the CUDA error text available from
+ * msp_last_error() (thread-local).  Empty inputs are legal (nrows == 0,
+ * nnz == 0, all rows empty).  Floating-point results accumulate in fp64
+ * and round once to the value type on store (reading Z4); SpAdd
+ * values are exact (one IEEE addition per matched pair).  Results are
+ * deterministic run to run (no floating-point atomics, fixed carry order).
+ */
+#ifndef MSP_H_
+#define MSP_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MSP_VERSION 1
+
+typedef enum {
+    MSP_OK = 0,
+    MSP_ERR_ARG = 1,         /* null pointer or negative size */
+    MSP_ERR_DTYPE = 2,       /* unsupported or mismatched value type */
+    MSP_ERR_SHAPE = 3,       /* A, B, x, y shapes incompatible */
+    MSP_ERR_WORKSPACE = 4,   /* workspace too small (query *_workspace) */
+    MSP_ERR_OVERFLOW = 5,    /* nnz(C) > INT32_MAX (int32 indices, Z16) */
+    MSP_ERR_INPUT = 6,       /* msp_csr_check found a malformed matrix */
+    MSP_ERR_CUDA = 7,        /* CUDA launch / runtime error, see msp_last_error */
+    MSP_ERR_NCCL = 8,        /* reserved for the multi-GPU layer */
+    MSP_ERR_UNSUPPORTED = 9  /* e.g. no sm_100 device */
+} msp_status;
+
+typedef enum { MSP_F32 = 0, MSP_F64 = 1 } msp_dtype;
+
+typedef struct {
+    int32_t nrows;
+    int32_t ncols;
+    int64_t nnz;                 /* must equal row_offsets[nrows] */
+    const int32_t *row_offsets;  /* device, [nrows+1] */
+    const int32_t *col_idx;      /* device, [nnz] */
+    const void *vals;            /* device, [nnz] of dtype */
+    int32_t dtype;               /* msp_dtype */
+} msp_csr;
+
+/* Human-readable name of a status code (static string). */
+const char *msp_status_string(int status);
+/* Detail of the last error raised on the calling host thread ("" if none). */
+const char *msp_last_error(void);
+/* MSP_VERSION of the loaded library. */
+int msp_version(void);
+
+/* ------------------------------------------------------------------------
+ * SpMV  y = A x      (Section III-A)
+ *
+ * One persistent launch: each CTA takes an equal contiguous range of the
+ * merge path of row_end = row_offsets[1..nrows] with the nonzero indices
+ * (equal share of rows plus nonzeros), streams its tiles of
+ * col_idx/vals through shared memory with TMA bulk copies, gathers x,
+ * reduces by row in-tile and emits one (row, partial) carry
+ * per CTA; the last CTA to finish adds the carries in CTA order (the update
+ * phase; reading Z21).
+ *
+ * x: device [ncols] of A.dtype.  y: device [nrows] of A.dtype, written
+ * entirely (empty rows get +0.0).  ws: device workspace of at least
+ * msp_spmv_workspace() bytes, zero-filled before its first use.  Async.
+ * ------------------------------------------------------------------------ */
+msp_status msp_spmv_workspace(const msp_csr *A, size_t *bytes);
+msp_status msp_spmv(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes,
+                    void *stream);
+
+/* ------------------------------------------------------------------------
+ * SpAdd  C = A + B   (P:496-550 union of (row,col) tuples in Algorithm 1
+ * order P:476-490; balanced path P:686-790; two phases P:816-838)
+ *
+ * A and B: same shape and dtype, sorted unique columns per row.
+ * Symbolic: counts the unique tuples of every row of C (cancellations keep
+ * an explicit zero, reading Z1), writes C_row_offsets (device int32
+ * [nrows+1]) and returns nnz(C) in *nnzC_host; synchronises the stream.
+ * Returns MSP_ERR_OVERFLOW if nnz(C) > INT32_MAX.
+ * Numeric: fills C_col_idx (device int32 [nnzC]) and C_vals (device
+ * [nnzC] of dtype); a matched pair gives (T)(a + b), A's value first
+ * (Alg. 1 tie order).  Uses the partition the symbolic call stored in ws.
+ * Async.
+ * ------------------------------------------------------------------------ */
+msp_status msp_spadd_workspace(const msp_csr *A, const msp_csr *B, size_t *bytes);
+msp_status msp_spadd_symbolic(const msp_csr *A, const msp_csr *B, int32_t *C_row_offsets,
+                              int64_t *nnzC_host, void *ws, size_t ws_bytes, void *stream);
+msp_status msp_spadd_numeric(const msp_csr *A, const msp_csr *B, const int32_t *C_row_offsets,
+                             int32_t *C_col_idx, void *C_vals, void *ws, size_t ws_bytes,
+                             void *stream);
+
+/* ------------------------------------------------------------------------
+ * SpGEMM  C = A B    (ESC: expansion, sorting, compression, P:256-262,
+ * P:840-1212, Section III-C)
+ *
+ * Setup: S = exclusive prefix sum (int64) of the B row lengths
+ * referenced by A's column indices, Nprods = S[nnzA], the COO row of every
+ * A nonzero, and the classification of rows whose product count exceeds
+ * one tile.  Returns the sizes in *info_host and synchronises.
+ * Symbolic: products are partitioned into tiles by a merge-path search over
+ * (S, product index) (reading Z7), expanded, sorted by
+ * (row, col) with a block merge sort and compressed; rows that straddle a
+ * tile boundary and rows longer than a tile are completed by a second pass
+ * (the paper's global phase).  Writes C_row_offsets and
+ * *nnzC_host; synchronises.  MSP_ERR_OVERFLOW if nnz(C) > INT32_MAX.
+ * Numeric: same passes with values; writes C_col_idx / C_vals; fp64
+ * accumulation in product order (k ascending).  Async.
+ * setup_ws: msp_spgemm_setup_workspace() bytes; main_ws: info.main_ws_bytes.
+ * ------------------------------------------------------------------------ */
+typedef struct {
+    int64_t nprods;          /* sum over A nonzeros of nnz(B row col) */
+    int64_t ntiles;          /* product tiles of the main pass */
+    int64_t long_rows;       /* rows with more products than one tile */
+    int64_t long_products;   /* products in those rows */
+    int64_t max_row_products;
+    int64_t main_ws_bytes;   /* size of the main workspace */
+} msp_spgemm_info;
+
+msp_status msp_spgemm_setup_workspace(const msp_csr *A, const msp_csr *B, size_t *bytes);
+msp_status msp_spgemm_setup(const msp_csr *A, const msp_csr *B, void *setup_ws,
+                            size_t setup_ws_bytes, msp_spgemm_info *info_host, void *stream);
+msp_status msp_spgemm_symbolic(const msp_csr *A, const msp_csr *B, const void *setup_ws,
+                               size_t setup_ws_bytes, void *main_ws, size_t main_ws_bytes,
+                               int32_t *C_row_offsets, int64_t *nnzC_host, void *stream);
+msp_status msp_spgemm_numeric(const msp_csr *A, const msp_csr *B, const void *setup_ws,
+                              size_t setup_ws_bytes, void *main_ws, size_t main_ws_bytes,
+                              const int32_t *C_row_offsets, int32_t *C_col_idx, void *C_vals,
+                              void *stream);
+
+/* ------------------------------------------------------------------------
+ * Input validation (the CSR contract of P:316-322).
+ * flags_host receives a bit set: 1 = row_offsets not monotone or
+ * row_offsets[0] != 0 or row_offsets[nrows] != nnz, 2 = column out of
+ * [0, ncols), 4 = columns not strictly increasing within a row (only
+ * checked when require_sorted_unique != 0).  Returns MSP_ERR_INPUT if any
+ * flag is set.  ws: at least 16 bytes, zero-filled.  Synchronises.
+ * ------------------------------------------------------------------------ */
+msp_status msp_csr_check(const msp_csr *A, int require_sorted_unique, int32_t *flags_host,
+                         void *ws, size_t ws_bytes, void *stream);
+
+/* ------------------------------------------------------------------------
+ * Multi-GPU helpers.  Row blocks are balanced by nnz:
+ * rank r owns rows [R_r, R_{r+1}), R_r = lower_bound(row_offsets,
+ * ceil(r * nnz / P)), R_0 = 0, R_P = nrows.  row_offsets_host is a HOST
+ * array [nrows+1]; row_starts_host a HOST array [P+1].  Pure host code.
+ * ------------------------------------------------------------------------ */
+msp_status msp_row_split(const int32_t *row_offsets_host, int32_t nrows, int32_t P,
+                         int32_t *row_starts_host);
+
+/* Rebase a row-offset array on the device: out[i] = in[i] - in[0] + base,
+ * i in [0, n); `in` and `out` must not alias.  Used to form row-block views
+ * and to concatenate gathered blocks.  Async. */
+msp_status msp_rebase_offsets(const int32_t *in, int32_t *out, int64_t n, int64_t base,
+                              void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MSP_H_ */

@@ -1,0 +1,289 @@
+// api.cu -- the extern "C" boundary of libmsp (include/msp.h).
+//
+// Host-side argument, shape and dtype validation happens here, before any
+// launch; the kernels live in spmv.cu / spadd.cu / spgemm.cu / scan.cu /
+// check.cu.  No call allocates device memory: every buffer is the caller's.
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+
+#include "internal.h"
+
+namespace msp {
+
+static thread_local char g_err[512] = "";
+
+void set_error(const char *fmt, ...)
+{
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+}
+
+void clear_error() { g_err[0] = 0; }
+
+msp_status cuda_check(cudaError_t e, const char *where)
+{
+    if (e == cudaSuccess) return MSP_OK;
+    set_error("%s: %s (%s)", where, cudaGetErrorString(e), cudaGetErrorName(e));
+    return MSP_ERR_CUDA;
+}
+
+msp_status last_launch(const char *where) { return cuda_check(cudaGetLastError(), where); }
+
+int sm_count()
+{
+    static int cache[64] = {0};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return 148;
+    if (dev < 0 || dev >= 64) return 148;
+    if (!cache[dev]) {
+        int n = 0;
+        if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
+        cache[dev] = n;
+    }
+    return cache[dev];
+}
+
+}  // namespace msp
+
+using namespace msp;
+
+namespace {
+
+msp_status check_csr(const msp_csr *A, const char *name)
+{
+    if (!A) {
+        set_error("%s is NULL", name);
+        return MSP_ERR_ARG;
+    }
+    if (A->nrows < 0 || A->ncols < 0 || A->nnz < 0) {
+        set_error("%s: negative size", name);
+        return MSP_ERR_ARG;
+    }
+    if (A->nnz > INT32_MAX) {
+        set_error("%s: nnz exceeds int32 indices", name);
+        return MSP_ERR_OVERFLOW;
+    }
+    if (A->dtype != MSP_F32 && A->dtype != MSP_F64) {
+        set_error("%s: dtype %d not supported", name, int(A->dtype));
+        return MSP_ERR_DTYPE;
+    }
+    if (!A->row_offsets || (A->nnz > 0 && (!A->col_idx || !A->vals))) {
+        set_error("%s: NULL array", name);
+        return MSP_ERR_ARG;
+    }
+    return MSP_OK;
+}
+
+inline cudaStream_t as_stream(void *s) { return static_cast<cudaStream_t>(s); }
+
+}  // namespace
+
+extern "C" {
+
+const char *msp_status_string(int status)
+{
+    switch (status) {
+    case MSP_OK: return "MSP_OK";
+    case MSP_ERR_ARG: return "MSP_ERR_ARG";
+    case MSP_ERR_DTYPE: return "MSP_ERR_DTYPE";
+    case MSP_ERR_SHAPE: return "MSP_ERR_SHAPE";
+    case MSP_ERR_WORKSPACE: return "MSP_ERR_WORKSPACE";
+    case MSP_ERR_OVERFLOW: return "MSP_ERR_OVERFLOW";
+    case MSP_ERR_INPUT: return "MSP_ERR_INPUT";
+    case MSP_ERR_CUDA: return "MSP_ERR_CUDA";
+    case MSP_ERR_NCCL: return "MSP_ERR_NCCL";
+    case MSP_ERR_UNSUPPORTED: return "MSP_ERR_UNSUPPORTED";
+    default: return "MSP_ERR_UNKNOWN";
+    }
+}
+
+const char *msp_last_error(void) { return g_err; }
+
+int msp_version(void) { return MSP_VERSION; }
+
+// ------------------------------------------------------------------ SpMV
+msp_status msp_spmv_workspace(const msp_csr *A, size_t *bytes)
+{
+    clear_error();
+    msp_status st = check_csr(A, "A");
+    if (st != MSP_OK) return st;
+    if (!bytes) return MSP_ERR_ARG;
+    *bytes = spmv_ws_bytes(A);
+    return MSP_OK;
+}
+
+msp_status msp_spmv(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, void *stream)
+{
+    clear_error();
+    msp_status st = check_csr(A, "A");
+    if (st != MSP_OK) return st;
+    if ((A->ncols > 0 && !x) || (A->nrows > 0 && !y) || !ws) {
+        set_error("spmv: NULL x, y or workspace");
+        return MSP_ERR_ARG;
+    }
+    if (ws_bytes < spmv_ws_bytes(A)) {
+        set_error("spmv: workspace %zu < %zu bytes", ws_bytes, spmv_ws_bytes(A));
+        return MSP_ERR_WORKSPACE;
+    }
+    return spmv_run(A, x, y, ws, ws_bytes, as_stream(stream));
+}
+
+// ------------------------------------------------------------------ SpAdd
+static msp_status check_pair_add(const msp_csr *A, const msp_csr *B)
+{
+    msp_status st = check_csr(A, "A");
+    if (st == MSP_OK) st = check_csr(B, "B");
+    if (st != MSP_OK) return st;
+    if (A->nrows != B->nrows || A->ncols != B->ncols) {
+        set_error("spadd: shapes %dx%d and %dx%d differ", A->nrows, A->ncols, B->nrows, B->ncols);
+        return MSP_ERR_SHAPE;
+    }
+    if (A->dtype != B->dtype) {
+        set_error("spadd: dtypes differ");
+        return MSP_ERR_DTYPE;
+    }
+    return MSP_OK;
+}
+
+msp_status msp_spadd_workspace(const msp_csr *A, const msp_csr *B, size_t *bytes)
+{
+    clear_error();
+    msp_status st = check_pair_add(A, B);
+    if (st != MSP_OK) return st;
+    if (!bytes) return MSP_ERR_ARG;
+    *bytes = spadd_ws_bytes(A, B);
+    return MSP_OK;
+}
+
+msp_status msp_spadd_symbolic(const msp_csr *A, const msp_csr *B, int32_t *C_row_offsets, int64_t *nnzC_host,
+                              void *ws, size_t ws_bytes, void *stream)
+{
+    clear_error();
+    msp_status st = check_pair_add(A, B);
+    if (st != MSP_OK) return st;
+    if (!C_row_offsets || !nnzC_host || !ws) return MSP_ERR_ARG;
+    if (ws_bytes < spadd_ws_bytes(A, B)) return MSP_ERR_WORKSPACE;
+    return spadd_symbolic_run(A, B, C_row_offsets, nnzC_host, ws, ws_bytes, as_stream(stream));
+}
+
+msp_status msp_spadd_numeric(const msp_csr *A, const msp_csr *B, const int32_t *C_row_offsets, int32_t *C_col_idx,
+                             void *C_vals, void *ws, size_t ws_bytes, void *stream)
+{
+    clear_error();
+    msp_status st = check_pair_add(A, B);
+    if (st != MSP_OK) return st;
+    if (!C_row_offsets || !ws) return MSP_ERR_ARG;
+    if (ws_bytes < spadd_ws_bytes(A, B)) return MSP_ERR_WORKSPACE;
+    return spadd_numeric_run(A, B, C_row_offsets, C_col_idx, C_vals, ws, ws_bytes, as_stream(stream));
+}
+
+// ------------------------------------------------------------------ SpGEMM
+static msp_status check_pair_mul(const msp_csr *A, const msp_csr *B)
+{
+    msp_status st = check_csr(A, "A");
+    if (st == MSP_OK) st = check_csr(B, "B");
+    if (st != MSP_OK) return st;
+    if (A->ncols != B->nrows) {
+        set_error("spgemm: A is %dx%d but B is %dx%d", A->nrows, A->ncols, B->nrows, B->ncols);
+        return MSP_ERR_SHAPE;
+    }
+    if (A->dtype != B->dtype) {
+        set_error("spgemm: dtypes differ");
+        return MSP_ERR_DTYPE;
+    }
+    return MSP_OK;
+}
+
+msp_status msp_spgemm_setup_workspace(const msp_csr *A, const msp_csr *B, size_t *bytes)
+{
+    clear_error();
+    msp_status st = check_pair_mul(A, B);
+    if (st != MSP_OK) return st;
+    if (!bytes) return MSP_ERR_ARG;
+    *bytes = spgemm_setup_ws_bytes(A, B);
+    return MSP_OK;
+}
+
+msp_status msp_spgemm_setup(const msp_csr *A, const msp_csr *B, void *setup_ws, size_t setup_ws_bytes,
+                            msp_spgemm_info *info_host, void *stream)
+{
+    clear_error();
+    msp_status st = check_pair_mul(A, B);
+    if (st != MSP_OK) return st;
+    if (!setup_ws || !info_host) return MSP_ERR_ARG;
+    if (setup_ws_bytes < spgemm_setup_ws_bytes(A, B)) return MSP_ERR_WORKSPACE;
+    return spgemm_setup_run(A, B, setup_ws, setup_ws_bytes, info_host, as_stream(stream));
+}
+
+msp_status msp_spgemm_symbolic(const msp_csr *A, const msp_csr *B, const void *setup_ws, size_t setup_ws_bytes,
+                               void *main_ws, size_t main_ws_bytes, int32_t *C_row_offsets, int64_t *nnzC_host,
+                               void *stream)
+{
+    clear_error();
+    msp_status st = check_pair_mul(A, B);
+    if (st != MSP_OK) return st;
+    if (!setup_ws || !main_ws || !C_row_offsets || !nnzC_host) return MSP_ERR_ARG;
+    return spgemm_symbolic_run(A, B, setup_ws, setup_ws_bytes, main_ws, main_ws_bytes, C_row_offsets, nnzC_host,
+                               as_stream(stream));
+}
+
+msp_status msp_spgemm_numeric(const msp_csr *A, const msp_csr *B, const void *setup_ws, size_t setup_ws_bytes,
+                              void *main_ws, size_t main_ws_bytes, const int32_t *C_row_offsets,
+                              int32_t *C_col_idx, void *C_vals, void *stream)
+{
+    clear_error();
+    msp_status st = check_pair_mul(A, B);
+    if (st != MSP_OK) return st;
+    if (!setup_ws || !main_ws || !C_row_offsets) return MSP_ERR_ARG;
+    return spgemm_numeric_run(A, B, setup_ws, setup_ws_bytes, main_ws, main_ws_bytes, C_row_offsets, C_col_idx,
+                              C_vals, as_stream(stream));
+}
+
+// ------------------------------------------------------------------ misc
+msp_status msp_csr_check(const msp_csr *A, int require_sorted_unique, int32_t *flags_host, void *ws,
+                         size_t ws_bytes, void *stream)
+{
+    clear_error();
+    msp_status st = check_csr(A, "A");
+    if (st != MSP_OK) return st;
+    if (!ws) return MSP_ERR_ARG;
+    return csr_check_run(A, require_sorted_unique, flags_host, ws, ws_bytes, as_stream(stream));
+}
+
+msp_status msp_row_split(const int32_t *rp, int32_t nrows, int32_t P, int32_t *starts)
+{
+    clear_error();
+    if (!rp || !starts || nrows < 0 || P < 1) return MSP_ERR_ARG;
+    const int64_t nnz = rp[nrows];
+    starts[0] = 0;
+    for (int32_t r = 1; r < P; ++r) {
+        const int64_t target = (int64_t(r) * nnz + P - 1) / P;
+        // lower_bound(rp[0..nrows], target)
+        int32_t lo = 0, hi = nrows;
+        while (lo < hi) {
+            const int32_t mid = lo + (hi - lo) / 2;
+            if (int64_t(rp[mid]) < target) lo = mid + 1;
+            else hi = mid;
+        }
+        starts[r] = lo;
+    }
+    starts[P] = nrows;
+    return MSP_OK;
+}
+
+msp_status msp_rebase_offsets(const int32_t *in, int32_t *out, int64_t n, int64_t base, void *stream)
+{
+    clear_error();
+    if (n < 0 || (n > 0 && (!in || !out))) return MSP_ERR_ARG;
+    if (in == out && n > 0) {
+        set_error("rebase: in and out alias");
+        return MSP_ERR_ARG;
+    }
+    return rebase_run(in, out, n, base, as_stream(stream));
+}
+
+}  // extern "C"

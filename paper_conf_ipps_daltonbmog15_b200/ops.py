@@ -1,0 +1,248 @@
+"""PyTorch-facing wrappers of the libmsp C ABI (argument marshalling only).
+
+Tensors live on a CUDA device; outputs and workspaces are allocated with
+torch and passed to libmsp by pointer together with the current CUDA stream.
+Every computation happens in the sm_100a kernels of libmsp.so; there is no
+CPU path.  Names follow the paper: spmv (Section III-A), spadd (III-B),
+spgemm (III-C).
+"""
+from __future__ import annotations
+
+import ctypes
+from dataclasses import dataclass
+
+import torch
+
+from ._lib import MSP_F32, MSP_F64, check, lib, msp_csr, msp_spgemm_info
+
+_DT = {torch.float32: MSP_F32, torch.float64: MSP_F64}
+
+
+@dataclass
+class CsrTensor:
+    """CSR matrix on a CUDA device: row_offsets int32[m+1], col_idx int32[nnz],
+    vals float32/float64[nnz]; columns sorted within each row."""
+    rp: torch.Tensor
+    col: torch.Tensor
+    val: torch.Tensor
+    shape: tuple[int, int]
+
+    @property
+    def nnz(self) -> int:
+        return int(self.col.numel())
+
+    @property
+    def dtype(self):
+        return self.val.dtype
+
+    @property
+    def device(self):
+        return self.val.device
+
+    @classmethod
+    def from_arrays(cls, rp, col, val, shape, device="cuda") -> "CsrTensor":
+        t = lambda a, dt=None: torch.as_tensor(a, dtype=dt, device=device).contiguous()  # noqa: E731
+        return cls(t(rp, torch.int32), t(col, torch.int32), t(val), (int(shape[0]), int(shape[1])))
+
+    def c(self) -> msp_csr:
+        if self.val.dtype not in _DT:
+            raise TypeError(f"unsupported dtype {self.val.dtype}")
+        for t in (self.rp, self.col, self.val):
+            if not t.is_contiguous():
+                raise ValueError("CSR arrays must be contiguous")
+        return msp_csr(self.shape[0], self.shape[1], self.nnz, self.rp.data_ptr(),
+                       self.col.data_ptr() if self.nnz else 0, self.val.data_ptr() if self.nnz else 0,
+                       _DT[self.val.dtype])
+
+    def numpy(self):
+        return (self.rp.cpu().numpy(), self.col.cpu().numpy(), self.val.cpu().numpy())
+
+
+# ----------------------------------------------------------------- workspaces
+
+_WS: dict = {}
+
+
+def workspace(nbytes: int, device, slot: str, stream=None) -> torch.Tensor:
+    """Zero-initialised byte workspace cached per (device, stream, slot).  Each
+    slot is only ever used by one kind of call, whose kernels leave their
+    counters zeroed, so reuse needs no re-clearing."""
+    dev = torch.device(device)
+    s = stream if stream is not None else torch.cuda.current_stream(dev)
+    key = (dev.index, s.cuda_stream, slot)
+    buf = _WS.get(key)
+    if buf is None or buf.numel() < nbytes:
+        buf = torch.zeros(max(int(nbytes), 256), dtype=torch.uint8, device=dev)
+        _WS[key] = buf
+    return buf
+
+
+def _stream_ptr(device, stream=None):
+    s = stream if stream is not None else torch.cuda.current_stream(torch.device(device))
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+# ----------------------------------------------------------------- SpMV
+
+def spmv_workspace_bytes(A: CsrTensor) -> int:
+    n = ctypes.c_size_t(0)
+    a = A.c()
+    check("msp_spmv_workspace", lib().msp_spmv_workspace(ctypes.byref(a), ctypes.byref(n)))
+    return int(n.value)
+
+
+def spmv(A: CsrTensor, x: torch.Tensor, out: torch.Tensor | None = None, stream=None,
+         ws: torch.Tensor | None = None) -> torch.Tensor:
+    """y = A x  (merge-path SpMV)."""
+    if x.dtype != A.dtype or x.device != A.device or x.numel() != A.shape[1] or not x.is_contiguous():
+        raise ValueError("x must be a contiguous vector of A.dtype on A.device with A.shape[1] entries")
+    y = out if out is not None else torch.empty(A.shape[0], dtype=A.dtype, device=A.device)
+    a = A.c()
+    if ws is None:
+        ws = workspace(spmv_workspace_bytes(A), A.device, "spmv", stream)
+    check("msp_spmv", lib().msp_spmv(ctypes.byref(a), x.data_ptr(), y.data_ptr(), ws.data_ptr(),
+                                     ws.numel(), _stream_ptr(A.device, stream)))
+    return y
+
+
+# ----------------------------------------------------------------- SpAdd
+
+class SpAddPlan:
+    """Two-phase SpAdd: symbolic() counts C's rows and returns
+    nnz(C); numeric() fills C with the partition symbolic() stored."""
+
+    def __init__(self, A: CsrTensor, B: CsrTensor, stream=None):
+        self.A, self.B, self.stream = A, B, stream
+        self.a, self.b = A.c(), B.c()
+        n = ctypes.c_size_t(0)
+        check("msp_spadd_workspace", lib().msp_spadd_workspace(ctypes.byref(self.a), ctypes.byref(self.b),
+                                                               ctypes.byref(n)))
+        self.ws = workspace(int(n.value), A.device, "spadd", stream)
+        self.rp = torch.empty(A.shape[0] + 1, dtype=torch.int32, device=A.device)
+        self.nnz = None
+
+    def symbolic(self) -> int:
+        nnz = ctypes.c_int64(0)
+        check("msp_spadd_symbolic",
+              lib().msp_spadd_symbolic(ctypes.byref(self.a), ctypes.byref(self.b), self.rp.data_ptr(),
+                                       ctypes.byref(nnz), self.ws.data_ptr(), self.ws.numel(),
+                                       _stream_ptr(self.A.device, self.stream)))
+        self.nnz = int(nnz.value)
+        return self.nnz
+
+    def numeric(self, col: torch.Tensor | None = None, val: torch.Tensor | None = None) -> CsrTensor:
+        if self.nnz is None:
+            self.symbolic()
+        dev = self.A.device
+        col = col if col is not None else torch.empty(self.nnz, dtype=torch.int32, device=dev)
+        val = val if val is not None else torch.empty(self.nnz, dtype=self.A.dtype, device=dev)
+        check("msp_spadd_numeric",
+              lib().msp_spadd_numeric(ctypes.byref(self.a), ctypes.byref(self.b), self.rp.data_ptr(),
+                                      col.data_ptr() if self.nnz else None, val.data_ptr() if self.nnz else None,
+                                      self.ws.data_ptr(), self.ws.numel(), _stream_ptr(dev, self.stream)))
+        return CsrTensor(self.rp, col, val, self.A.shape)
+
+
+def spadd(A: CsrTensor, B: CsrTensor, stream=None) -> CsrTensor:
+    """C = A + B (balanced-path union)."""
+    p = SpAddPlan(A, B, stream)
+    p.symbolic()
+    return p.numeric()
+
+
+# ----------------------------------------------------------------- SpGEMM
+
+class SpGemmPlan:
+    """ESC SpGEMM: setup() -> Nprods and sizes, symbolic() ->
+    C.row_offsets and nnz(C), numeric() -> C.col / C.vals."""
+
+    def __init__(self, A: CsrTensor, B: CsrTensor, stream=None):
+        if A.shape[1] != B.shape[0]:
+            raise ValueError("inner dimensions differ")
+        self.A, self.B, self.stream = A, B, stream
+        self.a, self.b = A.c(), B.c()
+        n = ctypes.c_size_t(0)
+        check("msp_spgemm_setup_workspace",
+              lib().msp_spgemm_setup_workspace(ctypes.byref(self.a), ctypes.byref(self.b), ctypes.byref(n)))
+        self.ws1 = workspace(int(n.value), A.device, "spgemm_setup", stream)
+        self.info = None
+        self.ws2 = None
+        self.rp = torch.empty(A.shape[0] + 1, dtype=torch.int32, device=A.device)
+        self.nnz = None
+
+    def setup(self) -> msp_spgemm_info:
+        info = msp_spgemm_info()
+        check("msp_spgemm_setup",
+              lib().msp_spgemm_setup(ctypes.byref(self.a), ctypes.byref(self.b), self.ws1.data_ptr(),
+                                     self.ws1.numel(), ctypes.byref(info), _stream_ptr(self.A.device, self.stream)))
+        self.info = info
+        self.ws2 = workspace(int(info.main_ws_bytes), self.A.device, "spgemm_main", self.stream)
+        return info
+
+    @property
+    def nprods(self) -> int:
+        if self.info is None:
+            self.setup()
+        return int(self.info.nprods)
+
+    def symbolic(self) -> int:
+        if self.info is None:
+            self.setup()
+        nnz = ctypes.c_int64(0)
+        check("msp_spgemm_symbolic",
+              lib().msp_spgemm_symbolic(ctypes.byref(self.a), ctypes.byref(self.b), self.ws1.data_ptr(),
+                                        self.ws1.numel(), self.ws2.data_ptr(), self.ws2.numel(), self.rp.data_ptr(),
+                                        ctypes.byref(nnz), _stream_ptr(self.A.device, self.stream)))
+        self.nnz = int(nnz.value)
+        return self.nnz
+
+    def numeric(self, col: torch.Tensor | None = None, val: torch.Tensor | None = None) -> CsrTensor:
+        if self.nnz is None:
+            self.symbolic()
+        dev = self.A.device
+        col = col if col is not None else torch.empty(self.nnz, dtype=torch.int32, device=dev)
+        val = val if val is not None else torch.empty(self.nnz, dtype=self.A.dtype, device=dev)
+        check("msp_spgemm_numeric",
+              lib().msp_spgemm_numeric(ctypes.byref(self.a), ctypes.byref(self.b), self.ws1.data_ptr(),
+                                       self.ws1.numel(), self.ws2.data_ptr(), self.ws2.numel(), self.rp.data_ptr(),
+                                       col.data_ptr() if self.nnz else None, val.data_ptr() if self.nnz else None,
+                                       _stream_ptr(dev, self.stream)))
+        return CsrTensor(self.rp, col, val, (self.A.shape[0], self.B.shape[1]))
+
+
+def spgemm(A: CsrTensor, B: CsrTensor, stream=None) -> CsrTensor:
+    """C = A B (expand / sort / compress)."""
+    p = SpGemmPlan(A, B, stream)
+    p.setup()
+    p.symbolic()
+    return p.numeric()
+
+
+# ----------------------------------------------------------------- misc
+
+def csr_check(A: CsrTensor, sorted_unique: bool = True) -> int:
+    """Validate the CSR contract on the device; returns the flag bits."""
+    a = A.c()
+    ws = workspace(256, A.device, "check")
+    flags = ctypes.c_int32(0)
+    st = lib().msp_csr_check(ctypes.byref(a), int(sorted_unique), ctypes.byref(flags), ws.data_ptr(),
+                             ws.numel(), _stream_ptr(A.device))
+    if st not in (0, 6):
+        check("msp_csr_check", st)
+    return int(flags.value)
+
+
+def row_split(rp_host, P: int):
+    """nnz-balanced row blocks (host): R_r = lower_bound(rp, ceil(r nnz / P))."""
+    import numpy as np
+    rp = np.ascontiguousarray(rp_host, dtype=np.int32)
+    out = np.empty(P + 1, dtype=np.int32)
+    check("msp_row_split", lib().msp_row_split(rp.ctypes.data, rp.size - 1, P, out.ctypes.data))
+    return out
+
+
+def rebase_offsets(rp: torch.Tensor, base: int, out: torch.Tensor | None = None) -> torch.Tensor:
+    out = out if out is not None else torch.empty_like(rp)
+    check("msp_rebase_offsets", lib().msp_rebase_offsets(rp.data_ptr(), out.data_ptr(), rp.numel(), int(base),
+                                                         _stream_ptr(rp.device)))
+    return out
