@@ -91,10 +91,12 @@ __device__ __forceinline__ void named_bar_sync(int id, int nthreads)
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-// Plan of a TMA window copy: elements [lo, hi) of an array are placed in
-// shared memory so that each element keeps its address mod 16; the 16-byte
-// aligned interior goes through one bulk copy and at most 15 bytes at each
-// end are copied by plain loads (never touching memory outside [lo, hi)).
+// Plan of a TMA window copy of elements [lo, hi) of an array of `len`
+// elements: each element keeps its address mod 16 in shared memory.  The
+// window is widened to 16-byte boundaries (re-reading a few neighbouring
+// elements of the same array is harmless) so that it normally goes through
+// ONE bulk copy; only where widening would leave the array (a misaligned
+// base, or the array's last bytes) are up to 15 bytes copied by hand.
 struct WindowCopy {
     const char *bulk_src;  // null if no bulk part
     uint32_t bulk_bytes;
@@ -106,31 +108,40 @@ struct WindowCopy {
 };
 
 template <int ES>
-__device__ __forceinline__ WindowCopy plan_window(const void *base, int64_t lo, int64_t hi)
+__device__ __forceinline__ WindowCopy plan_window(const void *base, int64_t lo, int64_t hi, int64_t len)
 {
     WindowCopy w;
-    const uintptr_t s = reinterpret_cast<uintptr_t>(base) + uintptr_t(lo) * ES;
-    const uintptr_t e = reinterpret_cast<uintptr_t>(base) + uintptr_t(hi) * ES;
+    const uintptr_t b0 = reinterpret_cast<uintptr_t>(base);
+    const uintptr_t s = b0 + uintptr_t(lo) * ES;
+    const uintptr_t e = b0 + uintptr_t(hi) * ES;
+    const uintptr_t end = b0 + uintptr_t(len) * ES;
     const uintptr_t a_lo = s & ~uintptr_t(15);
-    uintptr_t b_lo = (s + 15) & ~uintptr_t(15);
-    uintptr_t b_hi = e & ~uintptr_t(15);
     w.first = uint32_t(s - a_lo);
+    w.head_elems = 0;
+    w.tail_elems = 0;
     if (hi <= lo) {
-        w.bulk_src = nullptr; w.bulk_bytes = 0; w.bulk_dst = 0;
-        w.head_elems = 0; w.tail_elems = 0; w.span = 16;
+        w.bulk_src = nullptr; w.bulk_bytes = 0; w.bulk_dst = 0; w.span = 16;
         return w;
     }
-    if (b_hi <= b_lo) {  // no aligned interior: everything by hand
-        w.bulk_src = nullptr; w.bulk_bytes = 0; w.bulk_dst = 0;
-        w.head_elems = uint32_t(hi - lo); w.tail_elems = 0;
-    } else {
+    uintptr_t b_lo = a_lo, b_hi = (e + 15) & ~uintptr_t(15);
+    if (b_lo < b0) {  // misaligned base: hand-copy up to the first aligned element
+        b_lo = (s + 15) & ~uintptr_t(15);
+        w.head_elems = uint32_t((b_lo < e ? b_lo - s : e - s) / ES);
+    }
+    if (b_hi > end) {  // array end: hand-copy the last partial 16 bytes
+        b_hi = e & ~uintptr_t(15);
+        if (b_hi < b_lo) b_hi = b_lo;
+        w.tail_elems = uint32_t((e - (b_hi > s ? b_hi : s)) / ES) ;
+        if (w.head_elems && b_hi <= b_lo) w.tail_elems = 0;  // head already covers [lo, hi)
+    }
+    if (b_hi > b_lo) {
         w.bulk_src = reinterpret_cast<const char *>(b_lo);
         w.bulk_bytes = uint32_t(b_hi - b_lo);
         w.bulk_dst = uint32_t(b_lo - a_lo);
-        w.head_elems = uint32_t((b_lo - s) / ES);
-        w.tail_elems = uint32_t((e - b_hi) / ES);
+    } else {
+        w.bulk_src = nullptr; w.bulk_bytes = 0; w.bulk_dst = 0;
     }
-    w.span = uint32_t(((e - a_lo) + 15) & ~uintptr_t(15));
+    w.span = uint32_t((((e + 15) & ~uintptr_t(15)) - a_lo));
     return w;
 }
 

@@ -31,6 +31,9 @@
 //   * fp32 inputs are promoted and accumulated in fp64 (reading Z4).
 #include <climits>
 #include <cstdio>
+#include <cstdlib>
+#include <algorithm>
+#include <type_traits>
 
 #include "common.cuh"
 #include "internal.h"
@@ -54,19 +57,38 @@ struct CtaRecord {  // one per CTA in the workspace
     double head_val;     // fp64 value written for head_row (before carries)
 };
 
-template <typename V, int NT_, int K_, int STAGES_>
+// NW worker warps of 32 lanes x K = 8 products each (one tile = NW * 256
+// merge items), plus one producer warp and one row warp.
+template <typename V, int NW_, int STAGES_, int RSLOTS_, int MINB_>
 struct Cfg {
-    static constexpr int NT = NT_;          // consumer threads
-    static constexpr int K = K_;            // products per consumer thread
+    static constexpr int NW = NW_;
+    static constexpr int K = 8;
+    static constexpr int WSPAN = 32 * K;                 // products per worker warp
+    static constexpr int T = NW * WSPAN;                 // merge items (rows + nonzeros) per tile
     static constexpr int STAGES = STAGES_;
-    static constexpr int NCW = NT / 32;
-    static constexpr int THREADS = NT + 32;
-    static constexpr int T = NT * K;        // merge items (rows + nonzeros) per tile
-    static constexpr int STAGE_BYTES = int(((4 + sizeof(V)) * T + 128 + 127) / 128 * 128);
-    static constexpr int PROD_BYTES = T * 8;
-    static constexpr int SMEM = STAGES * STAGE_BYTES + PROD_BYTES + 1024;
-    static_assert(K % 2 == 0 && K / 2 <= 8, "K must be even and <= 16");
+    static constexpr int MINB = MINB_;
+    static constexpr int THREADS = (NW + 2) * 32;
+    static constexpr int RING = STAGES_ + RSLOTS_ + 3;   // per-tile carry slots (> max warp skew)
+    static constexpr int DATA_BYTES = int(((4 + sizeof(V)) * T + 64 + 15) / 16 * 16);  // rp, col, val windows
+    static constexpr int FLAG_BYTES = T / 8;             // row-end bit per position
+    static constexpr int RMAP_BYTES = T * 2;             // row (tile-relative, +1) ending at a position
+    static constexpr int STAGE_BYTES = DATA_BYTES;       // TMA ring: released after phase A
+    static constexpr int RSLOTS = RSLOTS_;               // row-map ring: released after the walk
+    static constexpr int RSLOT_BYTES = FLAG_BYTES + RMAP_BYTES;
+    static constexpr int PROD_BYTES = NW * WSPAN * 8;    // warp-private product buffers
+    static constexpr int MISC_BYTES = 2048;
+    static constexpr int SMEM = STAGES * STAGE_BYTES + RSLOTS * RSLOT_BYTES + PROD_BYTES + MISC_BYTES;
 };
+
+__device__ __forceinline__ uint64_t gtimer()
+{
+    uint64_t t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+
+__device__ __forceinline__ int ld_volatile_s(const int *p) { return *reinterpret_cast<const volatile int *>(p); }
+__device__ __forceinline__ void st_volatile_s(int *p, int v) { *reinterpret_cast<volatile int *>(p) = v; }
 
 // 32-ary warp search on the CSR merge grid: smallest i in [lo, hi] with
 // NOT(rp[i+1] <= d - i - 1) (i.e. the number of row ends consumed before
@@ -95,25 +117,86 @@ __device__ __forceinline__ int warp_grid_search(const int32_t *__restrict__ rp, 
     return lo + __popc(__ballot_sync(0xffffffffu, pred));
 }
 
-template <typename V, class C>
-__global__ void __launch_bounds__(C::THREADS, 2)
-spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const int32_t *__restrict__ col,
-                  const V *__restrict__ val, const V *__restrict__ x, V *__restrict__ y,
-                  CtaRecord *__restrict__ recs, unsigned *__restrict__ counter)
+__device__ __forceinline__ void mbar_wait_backoff(uint64_t *bar, uint32_t parity)
 {
+    while (!mbar_try_wait(bar, parity)) {
+    }
+}
+
+__device__ __forceinline__ void prefetch_l2(const void *p, uint32_t bytes)
+{
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+
+// L2 prefetch of elements [lo, hi) of an array (16-byte aligned interior).
+template <int ES>
+__device__ __forceinline__ void prefetch_range(const void *base, int64_t lo, int64_t hi)
+{
+    if (hi <= lo) return;
+    const uintptr_t s = (reinterpret_cast<uintptr_t>(base) + uintptr_t(lo) * ES + 15) & ~uintptr_t(15);
+    const uintptr_t e = (reinterpret_cast<uintptr_t>(base) + uintptr_t(hi) * ES) & ~uintptr_t(15);
+    if (e > s) prefetch_l2(reinterpret_cast<const void *>(s), uint32_t(e - s));
+}
+
+// Split search with a guess: probe the 32 consecutive rows around `g` first
+// (one ballot round when the tile has about as many rows as the last one),
+// and fall back to the 32-ary search on the remaining range.
+__device__ __forceinline__ int warp_grid_search_guess(const int32_t *__restrict__ rp, int64_t d, int lo, int hi,
+                                                      int g, int lane)
+{
+    if (hi - lo <= 32) return warp_grid_search(rp, d, lo, hi, lane);
+    int base = g - 16;
+    base = max(lo, min(base, hi - 32));
+    const int64_t p = int64_t(base) + lane;
+    const bool pred = int64_t(__ldg(rp + p + 1)) <= d - p - 1;
+    const int c = __popc(__ballot_sync(0xffffffffu, pred));
+    if (c > 0 && c < 32) return base + c;
+    if (c == 0) return (base == lo) ? lo : warp_grid_search(rp, d, lo, base, lane);
+    return warp_grid_search(rp, d, base + 32, hi, lane);
+}
+
+// Product buffer layout: logical position q (one fp64 product) lives in
+// 16-byte chunk c = q/2 at physical chunk c ^ ((c >> 3) & (K/2 - 1)), so that
+// both the strided writes of phase A and the K-consecutive reads of the walk
+// are bank-conflict free.
+template <int K>
+__device__ __forceinline__ int swz(int q)
+{
+    const int c = q >> 1;
+    return ((c ^ ((c >> 3) & (K / 2 - 1))) << 1) | (q & 1);
+}
+
+template <typename V, class C>
+__global__ void __launch_bounds__(C::THREADS, C::MINB)
+spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const int32_t *__restrict__ col,
+                  const V *__restrict__ val, const V *__restrict__ x, V *__restrict__ y, int32_t n_cols,
+                  CtaRecord *__restrict__ recs, unsigned *__restrict__ counter, int dbg_mode, void *dbg_ts)
+{
+    constexpr int K = C::K, NW = C::NW, WSPAN = C::WSPAN, RING = C::RING;
+    constexpr int FW = C::T / 32;  // flag words per tile
     extern __shared__ __align__(128) char smem[];
     char *stages = smem;
-    double *prod = reinterpret_cast<double *>(smem + C::STAGES * C::STAGE_BYTES);
-    char *misc = smem + C::STAGES * C::STAGE_BYTES + C::PROD_BYTES;
-    uint64_t *full = reinterpret_cast<uint64_t *>(misc);                 // [STAGES]
-    uint64_t *empty = full + C::STAGES;                                  // [STAGES]
-    TileMeta *meta = reinterpret_cast<TileMeta *>(empty + C::STAGES);    // [STAGES]
-    SegPair<double> *scan_w = reinterpret_cast<SegPair<double> *>(meta + C::STAGES);  // [NCW]
+    char *rslots = smem + C::STAGES * C::STAGE_BYTES;                   // [RSLOTS] flags + row map
+    double *prodbuf = reinterpret_cast<double *>(rslots + C::RSLOTS * C::RSLOT_BYTES);  // [NW][WSPAN]
+    char *misc = reinterpret_cast<char *>(prodbuf) + C::PROD_BYTES;
+    uint64_t *full = reinterpret_cast<uint64_t *>(misc);               // [STAGES] TMA landed
+    uint64_t *empty = full + C::STAGES;                                // [STAGES] stage free
+    uint64_t *rowsrdy = empty + C::STAGES;                             // [RSLOTS] row map built
+    uint64_t *rowsfree = rowsrdy + C::RSLOTS;                          // [RSLOTS] row map consumed
+    TileMeta *meta = reinterpret_cast<TileMeta *>(rowsfree + C::RSLOTS);  // [STAGES]
+    double *agg_v = reinterpret_cast<double *>(meta + C::STAGES);     // [RING][NW] warp trailing sums
+    double *cta_v = agg_v + RING * NW;                                 // [RING] carry leaving each tile
+    int *agg_f = reinterpret_cast<int *>(cta_v + RING);                // [RING][NW] warp had a row end
+    int *agg_seq = agg_f + RING * NW;                                  // [RING][NW] tile tag (t+1) once published
+    int *cta_f = agg_seq + RING * NW;                                  // [RING]
+    int *cta_seq = cta_f + RING;                                       // [RING] tile tag once cta_v/f valid
+    int *pub_cnt = cta_seq + RING;                                     // [RING] warps published
     __shared__ int s_carry_key, s_head_row, s_last;
     __shared__ double s_head_val;
 
     const int tid = threadIdx.x;
     const int lane = tid & 31;
+    const int warp = tid >> 5;
     const int G = gridDim.x;
     const int64_t total = int64_t(m) + nnz;
     const int64_t d_begin = int64_t(blockIdx.x) * total / G;
@@ -123,44 +206,70 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
     if (tid == 0) {
         for (int s = 0; s < C::STAGES; ++s) {
             mbar_init(&full[s], 1);
-            mbar_init(&empty[s], 1);
+            mbar_init(&empty[s], NW + 1);
+        }
+        for (int s = 0; s < C::RSLOTS; ++s) {
+            mbar_init(&rowsrdy[s], 1);
+            mbar_init(&rowsfree[s], NW);
         }
         fence_mbar_init();
         s_carry_key = -1;
         s_head_row = -1;
         s_head_val = 0.0;
     }
+    for (int i = tid; i < RING * NW; i += blockDim.x) agg_seq[i] = 0;
+    for (int i = tid; i < RING; i += blockDim.x) {
+        cta_seq[i] = 0;
+        pub_cnt[i] = 0;
+    }
     __syncthreads();
 
-    if (tid >= C::NT) {
+    if (warp == NW) {
         // ============================ producer warp ============================
         const uint64_t pol = policy_evict_first();
-        int i_s = warp_grid_search(rp, d_begin, int(max64(0, d_begin - nnz)),
-                                   int(min64(d_begin, m)), lane);
+        int i_s = warp_grid_search(rp, d_begin, int(max64(0, d_begin - nnz)), int(min64(d_begin, m)), lane);
         int j_s = int(d_begin - i_s);
+        int prev_rows = 0;
+        const int64_t j_cta_end = min64(nnz, d_end);  // upper bound for prefetching
+        if (lane == 0) {                               // warm the first two tiles' data in L2
+            prefetch_range<4>(rp, i_s, min64(int64_t(m) + 1, int64_t(i_s) + 2 * C::T + 1));
+            prefetch_range<4>(col, j_s, min64(j_cta_end, int64_t(j_s) + 2 * C::T));
+            prefetch_range<int(sizeof(V))>(val, j_s, min64(j_cta_end, int64_t(j_s) + 2 * C::T));
+        }
         for (int t = 0; t < ntiles; ++t) {
             const int stage = t % C::STAGES;
-            const int64_t de = min(d_begin + int64_t(t + 1) * C::T, d_end);
+            if ((dbg_mode & 16) && lane == 0 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 0] = gtimer();
+            const int64_t de = min64(d_begin + int64_t(t + 1) * C::T, d_end);
             const int lo = int(max64(i_s, de - nnz));
             const int hi = int(min64(m, de - j_s));
-            const int i_e = warp_grid_search(rp, de, lo, hi, lane);
+            const int i_e = warp_grid_search_guess(rp, de, lo, hi, i_s + prev_rows, lane);
             const int j_e = int(de - i_e);
-            if (t >= C::STAGES) mbar_wait(&empty[stage], ((t / C::STAGES) - 1) & 1);
+            if ((dbg_mode & 16) && lane == 0 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 1] = gtimer();
+            prev_rows = i_e - i_s;
+            if (lane == 0) {  // keep the data two tiles ahead streaming into L2
+                const int64_t rr = max(prev_rows, 32);
+                prefetch_range<4>(rp, int64_t(i_e) + rr, min64(int64_t(m) + 1, int64_t(i_e) + 3 * rr + 1));
+                prefetch_range<4>(col, int64_t(j_e) + C::T, min64(j_cta_end, int64_t(j_e) + 2 * C::T));
+                prefetch_range<int(sizeof(V))>(val, int64_t(j_e) + C::T, min64(j_cta_end, int64_t(j_e) + 2 * C::T));
+            }
+            if (t >= C::STAGES) mbar_wait_backoff(&empty[stage], ((t / C::STAGES) - 1) & 1);
+            if ((dbg_mode & 16) && lane == 0 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 2] = gtimer();
             char *sb = stages + size_t(stage) * C::STAGE_BYTES;
             const int wr_end = min(i_e + 1, m);
             // windows: rp[i_s .. wr_end] (inclusive), col/val[j_s .. j_e)
-            const WindowCopy wr = plan_window<4>(rp, i_s, int64_t(wr_end) + 1);
-            const WindowCopy wc = plan_window<4>(col, j_s, j_e);
-            const WindowCopy wv = plan_window<int(sizeof(V))>(val, j_s, j_e);
+            const WindowCopy wr = plan_window<4>(rp, i_s, int64_t(wr_end) + 1, int64_t(m) + 1);
+            const WindowCopy wc = plan_window<4>(col, j_s, j_e, nnz);
+            const WindowCopy wv = plan_window<int(sizeof(V))>(val, j_s, j_e, nnz);
             const uint32_t off_r = 0, off_c = wr.span, off_v = wr.span + wc.span;
-            // ragged ends by hand (lanes), then one lane arrives + issues bulk copies
             const int nr = int(wr.head_elems + wr.tail_elems);
             const int nc = int(wc.head_elems + wc.tail_elems);
             const int nv = int(wv.head_elems + wv.tail_elems);
-            if (lane < nr) window_manual<int32_t>(wr, rp, i_s, int64_t(wr_end) + 1, sb + off_r, lane);
-            else if (lane < nr + nc) window_manual<int32_t>(wc, col, j_s, j_e, sb + off_c, lane - nr);
-            else if (lane < nr + nc + nv) window_manual<V>(wv, val, j_s, j_e, sb + off_v, lane - nr - nc);
-            __syncwarp();
+            if (nr + nc + nv) {  // rare: misaligned base or the arrays' last bytes
+                if (lane < nr) window_manual<int32_t>(wr, rp, i_s, int64_t(wr_end) + 1, sb + off_r, lane);
+                else if (lane < nr + nc) window_manual<int32_t>(wc, col, j_s, j_e, sb + off_c, lane - nr);
+                else if (lane < nr + nc + nv) window_manual<V>(wv, val, j_s, j_e, sb + off_v, lane - nr - nc);
+                __syncwarp();
+            }
             if (lane == 0) {
                 TileMeta &mt = meta[stage];
                 mt.i_s = i_s; mt.i_e = i_e; mt.wr_end = wr_end;
@@ -176,123 +285,250 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             i_s = i_e;
             j_s = j_e;
         }
-    } else {
-        // ============================ consumers ================================
-        SegPair<double> carry{0, 0.0};  // running partial entering the next tile
+    } else if (warp == NW + 1) {
+        // ============================ row warp =================================
+        // Per tile: a row-end bit and the (tile-relative) row id at the
+        // position of every nonempty row's last nonzero; empty rows whose
+        // row-end item lies in the tile get y = +0.0 (Z6); the row holding the
+        // tile's last nonzero is the CTA carry key.
         for (int t = 0; t < ntiles; ++t) {
             const int stage = t % C::STAGES;
+            const int rs = t % C::RSLOTS;
             mbar_wait(&full[stage], (t / C::STAGES) & 1);
+            if (t >= C::RSLOTS) mbar_wait(&rowsfree[rs], ((t / C::RSLOTS) - 1) & 1);
             const TileMeta mt = meta[stage];
-            const char *sb = stages + size_t(stage) * C::STAGE_BYTES;
+            char *sb = stages + size_t(stage) * C::STAGE_BYTES;
             const int32_t *rps = reinterpret_cast<const int32_t *>(sb + mt.rp_first);  // rps[r - i_s] = rp[r]
-            const int32_t *cs = reinterpret_cast<const int32_t *>(sb + mt.col_first);
-            const V *vs = reinterpret_cast<const V *>(sb + mt.val_first);
-            const int z = mt.j_e - mt.j_s;
-
-            // ---- phase A: products in strided (coalesced) order ----
-            int cidx[C::K];
-#pragma unroll
-            for (int u = 0; u < C::K; ++u) {
-                const int q = tid + u * C::NT;
-                cidx[u] = (q < z) ? cs[q] : 0;
-            }
-            V xv[C::K];
-#pragma unroll
-            for (int u = 0; u < C::K; ++u) {
-                const int q = tid + u * C::NT;
-                xv[u] = (q < z) ? __ldg(x + cidx[u]) : V(0);
-            }
-#pragma unroll
-            for (int u = 0; u < C::K; ++u) {
-                const int q = tid + u * C::NT;
-                if (q < z) {
-                    const int c = q >> 1;
-                    const int phys = c ^ ((c >> 3) & (C::K / 2 - 1));
-                    prod[phys * 2 + (q & 1)] = double(vs[q]) * double(xv[u]);
-                }
-            }
-            // empty rows whose row-end item lies in this tile -> +0.0 (Z6)
-            for (int r = mt.i_s + tid; r < mt.i_e; r += C::NT)
-                if (rps[r - mt.i_s] == rps[r - mt.i_s + 1]) y[r] = V(0);
-            named_bar_sync(1, C::NT);
-
-            // ---- phase B: K consecutive products per thread, reduce by row ----
-            double p[C::K];
-#pragma unroll
-            for (int i = 0; i < C::K / 2; ++i) {
-                const int c = tid * (C::K / 2) + i;
-                const int phys = c ^ ((c >> 3) & (C::K / 2 - 1));
-                const double2 d2 = reinterpret_cast<const double2 *>(prod)[phys];
-                p[2 * i] = d2.x;
-                p[2 * i + 1] = d2.y;
-            }
-            const int qs = tid * C::K;
-            const int jfirst = mt.j_s + min(qs, z);
-            // row containing nonzero jfirst: first r with row_end[r] > jfirst
-            int lo = mt.i_s, hi = mt.wr_end;
-            while (lo < hi) {
-                const int mid = (lo + hi) >> 1;
-                if (rps[mid - mt.i_s + 1] > jfirst) hi = mid;
-                else lo = mid + 1;
-            }
-            int cur = lo;
-            int re = (cur < mt.wr_end) ? rps[cur - mt.i_s + 1] : INT_MAX;
-            double run = 0.0, fe_val = 0.0;
-            int fe_row = -1;
-            int emitted = 0;
-#pragma unroll
-            for (int k = 0; k < C::K; ++k) {
-                const int q = qs + k;
-                if (q < z) {
-                    run += p[k];
-                    const int jn = mt.j_s + q + 1;
-                    if (jn == re) {  // row `cur` ends after this nonzero
-                        if (!emitted) {
-                            fe_row = cur;
-                            fe_val = run;
-                            emitted = 1;
-                        } else {
-                            y[cur] = V(run);
+            uint32_t *flags = reinterpret_cast<uint32_t *>(rslots + size_t(rs) * C::RSLOT_BYTES);
+            uint16_t *rmap = reinterpret_cast<uint16_t *>(rslots + size_t(rs) * C::RSLOT_BYTES + C::FLAG_BYTES);
+            const int z = mt.j_e - mt.j_s, i_s = mt.i_s, j_s = mt.j_s;
+            for (int i = lane; i < FW; i += 32) flags[i] = 0u;
+            __syncwarp();
+            if ((dbg_mode & 3) != 1) {
+                for (int r = i_s + lane; r < mt.wr_end; r += 32) {
+                    const int a = rps[r - i_s] - j_s;
+                    const int b = rps[r - i_s + 1] - j_s;
+                    if (a == b) {
+                        if (r < mt.i_e) y[r] = V(0);
+                    } else {
+                        if (b > 0 && b <= z) {
+                            rmap[b - 1] = uint16_t(r - i_s + 1);
+                            atomicOr(&flags[(b - 1) >> 5], 1u << ((b - 1) & 31));
                         }
-                        run = 0.0;
-                        ++cur;
-                        re = (cur < mt.wr_end) ? rps[cur - mt.i_s + 1] : INT_MAX;
-                        if (re == jn) {  // skip empty rows (zero-filled separately)
-                            int l2 = cur + 1, h2 = mt.wr_end;
-                            while (l2 < h2) {
-                                const int mid = (l2 + h2) >> 1;
-                                if (rps[mid - mt.i_s + 1] > jn) h2 = mid;
-                                else l2 = mid + 1;
-                            }
-                            cur = l2;
-                            re = (cur < mt.wr_end) ? rps[cur - mt.i_s + 1] : INT_MAX;
-                        }
+                        if (z > 0 && a < z && b >= z) s_carry_key = (b > z) ? r : -1;
                     }
                 }
             }
-            SegPair<double> mine{emitted, run}, tot;
-            const SegPair<double> ex = block_seg_exclusive<double, C::NCW>(mine, carry, scan_w, 1, &tot);
-            if (tid == 0) mbar_arrive(&empty[stage]);  // stage fully consumed (scan barrier passed)
-            if (emitted) {
-                const double v = ex.v + fe_val;
-                y[fe_row] = V(v);
-                if (!ex.f) {  // first row this CTA emits: keep its fp64 value for the fix-up
-                    s_head_row = fe_row;
-                    s_head_val = v;
+            __syncwarp();
+            if (lane == 0) {
+                if ((dbg_mode & 16) && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 3] = gtimer();
+                mbar_arrive(&rowsrdy[rs]);
+                mbar_arrive(&empty[stage]);  // this warp no longer reads the stage
+            }
+        }
+    } else {
+        // ============================ worker warps =============================
+        // Worker `warp` owns products [warp*256, warp*256 + 256) of every tile.
+        //   phase A: lane l computes products l, l+32, ... (coalesced col/val
+        //            reads, x gathers of consecutive nonzeros) into a
+        //            warp-private swizzled buffer (P:444-456 strided -> blocked);
+        //   walk:    lane l sums products 8l .. 8l+7; at a row end it writes y
+        //            (its first row waits for the carry of earlier lanes);
+        //   scan:    warp segmented scan -> carry of earlier lanes; the warp's
+        //            first row also needs the carry of earlier warps / tiles,
+        //            read from their published trailing sums (look-back).
+        double *wprod = prodbuf + warp * WSPAN;
+        const int s_sw = (lane >> 1) & 3;
+        const unsigned col_lim = unsigned(n_cols);
+        const int wbase = warp * WSPAN;
+        int cidx[K];
+        V xv[K];
+        // phase A issue: columns from the stage, x gathers into registers.
+        // Positions >= z read other bytes of the stage (in bounds); their
+        // columns are clamped and their products masked in the walk.
+        V vv[K];
+        int nx_is = 0, nx_z = 0;  // row window start and nonzero count of the issued tile
+        auto a_issue = [&](int t) {
+            const int stage = t % C::STAGES;
+            mbar_wait(&full[stage], (t / C::STAGES) & 1);
+            if ((dbg_mode & 16) && lane == 0 && warp == 0 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 6] = gtimer();
+            nx_is = meta[stage].i_s;
+            nx_z = meta[stage].j_e - meta[stage].j_s;
+            const char *sb = stages + size_t(stage) * C::STAGE_BYTES;
+            const int32_t *cs = reinterpret_cast<const int32_t *>(sb + meta[stage].col_first) + wbase;
+            const V *vs = reinterpret_cast<const V *>(sb + meta[stage].val_first) + wbase;
+#pragma unroll
+            for (int u = 0; u < K; ++u) {
+                const unsigned c = unsigned(cs[lane + 32 * u]);
+                cidx[u] = int(c < col_lim ? c : 0u);
+            }
+#pragma unroll
+            for (int u = 0; u < K; ++u) xv[u] = __ldg(x + cidx[u]);
+#pragma unroll
+            for (int u = 0; u < K; ++u) vv[u] = vs[lane + 32 * u];
+        };
+        auto finish_first = [&](int r, double v0, int tt) {
+            const int sl = tt % RING;
+            double c = 0.0;
+            int f = 0;
+            for (int w2 = warp - 1; w2 >= 0 && !f; --w2) {
+                while (ld_volatile_s(&agg_seq[sl * NW + w2]) != tt + 1) {}
+                __threadfence_block();
+                c = reinterpret_cast<volatile double *>(agg_v)[sl * NW + w2] + c;
+                f = reinterpret_cast<volatile int *>(agg_f)[sl * NW + w2];
+            }
+            if (!f && tt > 0) {
+                const int ps = (tt - 1) % RING;
+                while (ld_volatile_s(&cta_seq[ps]) != tt) {}
+                __threadfence_block();
+                c = reinterpret_cast<volatile double *>(cta_v)[ps] + c;
+                f = reinterpret_cast<volatile int *>(cta_f)[ps];
+            }
+            const double v = v0 + c;
+            y[r] = V(v);
+            if (!f) {  // first row this CTA completes
+                s_head_row = r;
+                s_head_val = v;
+            }
+        };
+        int pend_r = -1, pend_t = 0;
+        double pend_v = 0.0;
+        a_issue(0);
+        for (int t = 0; t < ntiles; ++t) {
+            const int stage = t % C::STAGES;
+            const int slot = t % RING;
+            const int rs = t % C::RSLOTS;
+            const int tile_is = nx_is, z = nx_z;
+            // ---- phase A finish: products -> warp-private buffer ----
+#pragma unroll
+            for (int u = 0; u < K; ++u) wprod[swz<K>(lane + 32 * u)] = double(vv[u]) * double(xv[u]);
+            __syncwarp();
+            // the stage is released once the products are formed (releasing it
+            // right after the col/val loads measured slower: deeper TMA
+            // run-ahead raised memory contention and per-CTA tail variance)
+            if (lane == 0) mbar_arrive(&empty[stage]);
+            if ((dbg_mode & 16) && lane == 0 && warp == 0 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 4] = gtimer();
+            mbar_wait(&rowsrdy[rs], (t / C::RSLOTS) & 1);
+            if ((dbg_mode & 16) && lane == 0 && warp == 0 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 7] = gtimer();
+            if ((dbg_mode & 3) == 2) {  // profiling aid: phase A only
+                if (lane == 0) mbar_arrive(&rowsfree[rs]);
+                if (t + 1 < ntiles) a_issue(t + 1);
+                continue;
+            }
+            // ---- walk ----
+            const uint32_t *flags = reinterpret_cast<const uint32_t *>(rslots + size_t(rs) * C::RSLOT_BYTES);
+            const uint16_t *rmap =
+                reinterpret_cast<const uint16_t *>(rslots + size_t(rs) * C::RSLOT_BYTES + C::FLAG_BYTES);
+            const int qs = wbase + lane * K;  // tile position of this lane's first product
+            const unsigned mask = reinterpret_cast<const uint8_t *>(flags)[qs >> 3];
+            double run = 0.0, first_v = 0.0;
+            int first_r = -1;
+            if (qs < z) {
+                double p[K];
+                double *myp = wprod + lane * K;
+                if (qs + K <= z) {
+#pragma unroll
+                    for (int i = 0; i < K / 2; ++i) {
+                        const double2 d2 = reinterpret_cast<const double2 *>(myp)[i ^ s_sw];
+                        p[2 * i] = d2.x;
+                        p[2 * i + 1] = d2.y;
+                    }
+                } else {
+#pragma unroll
+                    for (int i = 0; i < K / 2; ++i) {
+                        const double2 d2 = reinterpret_cast<const double2 *>(myp)[i ^ s_sw];
+                        p[2 * i] = (qs + 2 * i < z) ? d2.x : 0.0;
+                        p[2 * i + 1] = (qs + 2 * i + 1 < z) ? d2.y : 0.0;
+                    }
+                }
+                double ev[K];
+#pragma unroll
+                for (int k = 0; k < K; ++k) {
+                    run += p[k];
+                    ev[k] = run;
+                    if ((mask >> k) & 1u) run = 0.0;
+                }
+                if (mask) {
+                    // row partials back into this lane's own product slots
+#pragma unroll
+                    for (int i = 0; i < K / 2; ++i)
+                        reinterpret_cast<double2 *>(myp)[i ^ s_sw] = make_double2(ev[2 * i], ev[2 * i + 1]);
+                    const int k0 = __ffs(mask) - 1;
+                    first_v = myp[(((k0 >> 1) ^ s_sw) << 1) | (k0 & 1)];
+                    first_r = tile_is + int(rmap[qs + k0]) - 1;
+                    for (unsigned rest = mask & (mask - 1); rest; rest &= rest - 1) {
+                        const int k = __ffs(rest) - 1;
+                        y[tile_is + int(rmap[qs + k]) - 1] = V(myp[(((k >> 1) ^ s_sw) << 1) | (k & 1)]);
+                    }
                 }
             }
-            if (tid == C::NT - 1) s_carry_key = (cur < mt.wr_end) ? cur : -1;
-            carry = tot;
+            const bool flagged = first_r >= 0;
+            // ---- warp segmented scan ----
+            const SegPair<double> inc = warp_seg_inclusive(SegPair<double>{flagged, run}, lane);
+            const double exv = __shfl_up_sync(0xffffffffu, inc.v, 1);
+            const unsigned fmask = __ballot_sync(0xffffffffu, flagged);
+            const int flane = fmask ? __ffs(fmask) - 1 : 32;
+            double pend_nv = 0.0;
+            if (flagged) {
+                const double v = lane ? first_v + exv : first_v;  // carry from earlier lanes
+                if (lane == flane) pend_nv = v;                    // also needs earlier warps' carry
+                else y[first_r] = V(v);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&rowsfree[rs]);  // done with this tile's row map
+            if ((dbg_mode & 16) && lane == 0 && warp == NW - 1 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 5] = gtimer();
+            // ---- publish this warp's trailing sum; the last warp of the tile
+            //      forms the carry leaving the tile ----
+            if (lane == 31) {
+                agg_v[slot * NW + warp] = inc.v;
+                agg_f[slot * NW + warp] = inc.f;
+                __threadfence_block();
+                st_volatile_s(&agg_seq[slot * NW + warp], t + 1);
+                const int done = atomicAdd(&pub_cnt[slot], 1);
+                if (done == NW - 1) {
+                    __threadfence_block();
+                    double c = 0.0;
+                    int f = 0;
+                    if (t > 0) {
+                        const int ps = (t - 1) % RING;
+                        while (ld_volatile_s(&cta_seq[ps]) != t) {}
+                        __threadfence_block();
+                        c = cta_v[ps];
+                        f = cta_f[ps];
+                    }
+                    for (int w2 = 0; w2 < NW; ++w2) {
+                        const int fw = reinterpret_cast<volatile int *>(agg_f)[slot * NW + w2];
+                        const double vw = reinterpret_cast<volatile double *>(agg_v)[slot * NW + w2];
+                        c = fw ? vw : c + vw;
+                        f |= fw;
+                    }
+                    cta_v[slot] = c;
+                    cta_f[slot] = f;
+                    pub_cnt[slot] = 0;
+                    __threadfence_block();
+                    st_volatile_s(&cta_seq[slot], t + 1);
+                }
+            }
+            // next tile's gathers fly while the previous tile's first row is finished
+            if (t + 1 < ntiles) a_issue(t + 1);
+            // ---- the warp's first row of tile t-1 (deferred one tile so that
+            //      the look-back never waits): carry of earlier warps (nearest
+            //      first), then of earlier tiles ----
+            if (pend_r >= 0) finish_first(pend_r, pend_v, pend_t);
+            pend_r = (lane == flane) ? first_r : -1;
+            pend_v = pend_nv;
+            pend_t = t;
         }
-        named_bar_sync(1, C::NT);
-        if (tid == 0) {
-            CtaRecord rec;
-            rec.carry_key = s_carry_key;
-            rec.carry_val = carry.v;
-            rec.head_row = s_head_row;
-            rec.head_val = s_head_val;
-            recs[blockIdx.x] = rec;
-        }
+        if (pend_r >= 0) finish_first(pend_r, pend_v, pend_t);
+    }
+    __syncthreads();
+    if (tid == 0) {
+        CtaRecord rec;
+        rec.carry_key = s_carry_key;
+        rec.carry_val = (ntiles > 0 && (dbg_mode & 3) == 0) ? cta_v[(ntiles - 1) % RING] : 0.0;
+        rec.head_row = s_head_row;
+        rec.head_val = s_head_val;
+        recs[blockIdx.x] = rec;
     }
 
     // ============================ update phase (last CTA) ======================
@@ -321,13 +557,53 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
     if (tid == 0) *counter = 0u;  // leave the workspace reusable
 }
 
-template <typename V>
-using SpmvCfg = Cfg<V, 256, 8, (sizeof(V) == 8 ? 3 : 4)>;
+// Tile shapes (consumer threads, products per thread, stages, CTAs/SM).
+// Config 0 is the default; MSP_SPMV_CFG=<n> selects another (tuning only).
+template <typename V, int I> struct Shape;
+template <typename V> struct Shape<V, 0> { using C = Cfg<V, 8, 2, 2, 2>; };
+template <typename V> struct Shape<V, 1> { using C = Cfg<V, 8, 2, 2, 3>; };
+template <typename V> struct Shape<V, 2> { using C = Cfg<V, 8, 3, 3, 2>; };
+template <typename V> struct Shape<V, 3> { using C = Cfg<V, 8, 2, 4, 2>; };
+template <typename V> struct Shape<V, 4> { using C = Cfg<V, 4, 2, 4, 4>; };
+constexpr int kNumShapes = 5;
 
-template <typename V>
-msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
+int debug_mode();
+int tiles_per_cta()
 {
-    using C = SpmvCfg<V>;
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("MSP_SPMV_TPC");
+        v = e ? atoi(e) : (1 << 30);  // default: one persistent wave
+        if (v < 2) v = 2;
+    }
+    return v;
+}
+void *g_dbg_ts = nullptr;
+}  // namespace
+void *g_dbg_ts_public() { return g_dbg_ts; }
+namespace {
+void *debug_ts()
+{
+    if (!g_dbg_ts && (debug_mode() & 16)) {
+        cudaMalloc(&g_dbg_ts, size_t(8192) * 256 * 8);  // profiling aid only
+        cudaMemset(g_dbg_ts, 0, size_t(8192) * 256 * 8);
+    }
+    return g_dbg_ts;
+}
+
+int debug_mode()
+{
+    static int d = -1;
+    if (d < 0) {
+        const char *e = getenv("MSP_SPMV_DEBUG");
+        d = e ? atoi(e) : 0;
+    }
+    return d;
+}
+
+template <typename V, class C>
+msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
+{
     auto kern = spmv_merge_kernel<V, C>;
     static int configured = 0;
     static int occ = 1;
@@ -335,33 +611,70 @@ msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_
         msp_status st = cuda_check(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM),
                                    "spmv: set smem");
         if (st != MSP_OK) return st;
+        st = cuda_check(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100),
+                        "spmv: carveout");
+        if (st != MSP_OK) return st;
         st = cuda_check(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, C::THREADS, C::SMEM),
                         "spmv: occupancy");
+        if (getenv("MSP_VERBOSE")) fprintf(stderr, "msp spmv: T=%d stages=%d smem=%d occupancy=%d CTAs/SM\n", C::T, C::STAGES, C::SMEM, occ);
         if (st != MSP_OK) return st;
         if (occ < 1) occ = 1;
+        if (occ > 4) occ = 4;
         configured = 1;
     }
-    const int64_t total = int64_t(A->nrows) + A->nnz;
     if (A->nrows == 0) return MSP_OK;
+    if (A->nnz == 0)  // every row is empty: y = +0.0 (Z6)
+        return cuda_check(cudaMemsetAsync(y, 0, size_t(A->nrows) * sizeof(V), s), "spmv: zero y");
+    const int64_t total = int64_t(A->nrows) + A->nnz;
     const int64_t ntiles = ceil_div(total, C::T);
-    const int64_t gmax = int64_t(occ) * sm_count();
-    const int grid = int(ntiles < gmax ? ntiles : gmax);
+    // Several waves of CTAs, each owning a contiguous range of about
+    // kTilesPerCta tiles: the hardware scheduler then balances CTAs that run
+    // slower than others, and a CTA's start-up search overlaps other CTAs.
+    const int64_t resident = int64_t(occ) * sm_count();
+    int64_t g = ceil_div(ntiles, tiles_per_cta());
+    if (g < resident) g = resident < ntiles ? resident : ntiles;
+    const int grid = int(g);
     Carve cv(ws, ws_bytes);
     unsigned *counter = cv.take<unsigned>(1);
     CtaRecord *recs = cv.take<CtaRecord>(size_t(grid));
     if (!cv.ok()) return MSP_ERR_WORKSPACE;
     kern<<<grid, C::THREADS, C::SMEM, s>>>(A->nrows, A->nnz, A->row_offsets, A->col_idx,
                                            static_cast<const V *>(A->vals), static_cast<const V *>(x),
-                                           static_cast<V *>(y), recs, counter);
+                                           static_cast<V *>(y), A->ncols, recs, counter, debug_mode(), debug_ts());
     return last_launch("spmv_merge_kernel");
+}
+
+int shape_choice()
+{
+    static int c = -1;
+    if (c < 0) {
+        const char *e = getenv("MSP_SPMV_CFG");
+        c = e ? atoi(e) : 0;
+        if (c < 0 || c >= kNumShapes) c = 0;
+    }
+    return c;
+}
+
+template <typename V>
+msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
+{
+    switch (shape_choice()) {
+    case 1: return launch_cfg<V, typename Shape<V, 1>::C>(A, x, y, ws, ws_bytes, s);
+    case 2: return launch_cfg<V, typename Shape<V, 2>::C>(A, x, y, ws, ws_bytes, s);
+    case 3: return launch_cfg<V, typename Shape<V, 3>::C>(A, x, y, ws, ws_bytes, s);
+    case 4: return launch_cfg<V, typename Shape<V, 4>::C>(A, x, y, ws, ws_bytes, s);
+    default: return launch_cfg<V, typename Shape<V, 0>::C>(A, x, y, ws, ws_bytes, s);
+    }
 }
 
 }  // namespace
 
-size_t spmv_ws_bytes(const msp_csr *)
+size_t spmv_ws_bytes(const msp_csr *A)
 {
-    // counter + one record per CTA; grid <= 4 CTAs per SM
-    return 256 + size_t(4) * size_t(sm_count()) * sizeof(CtaRecord) + 256;
+    // counter + one record per CTA (grid <= max(4 per SM, tiles / tiles-per-CTA))
+    const int64_t tiles = ceil_div(int64_t(A->nrows) + A->nnz, 1024);
+    const int64_t g = std::max<int64_t>(int64_t(4) * sm_count(), ceil_div(tiles, 2));
+    return 512 + size_t(g) * sizeof(CtaRecord);
 }
 
 msp_status spmv_run(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
@@ -371,3 +684,11 @@ msp_status spmv_run(const msp_csr *A, const void *x, void *y, void *ws, size_t w
 }
 
 }  // namespace msp
+
+// profiling aid (MSP_SPMV_DEBUG & 16): device buffer of per-tile timestamps
+extern "C" int msp_debug_copy_timestamps(void *host, size_t bytes)
+{
+    void *d = msp::g_dbg_ts_public();
+    if (!d) return -1;
+    return int(cudaMemcpy(host, d, bytes, cudaMemcpyDeviceToHost));
+}
