@@ -254,4 +254,26 @@ __device__ __forceinline__ T block_exclusive_sum(T v, T *smem_w, int bar_id, T *
     return lane == 0 ? wp : wp + ex;
 }
 
+// CTA-wide exclusive max over NW warps (named barrier); -1 before thread 0.
+template <int NW>
+__device__ __forceinline__ int block_exclusive_max(int v, int *smem_w, int bar_id)
+{
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    int inc = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int u = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc = max(inc, u);
+    }
+    if (lane == 31) smem_w[warp] = inc;
+    named_bar_sync(bar_id, NW * 32);
+    int wp = -1;
+#pragma unroll
+    for (int w = 0; w < NW; ++w)
+        if (w < warp) wp = max(wp, smem_w[w]);
+    const int ex = __shfl_up_sync(0xffffffffu, inc, 1);
+    named_bar_sync(bar_id, NW * 32);
+    return lane == 0 ? wp : max(wp, ex);
+}
+
 }  // namespace msp

@@ -46,6 +46,7 @@ size_t scan_ws_bytes(int64_t n);
 // out[i] = sum_{k<i} in[k] for i in [0, n]  (n+1 outputs; out[n] = total).
 msp_status scan_i32_to_i64(const int32_t *in, int64_t *out, int64_t n, void *ws, size_t ws_bytes,
                            cudaStream_t s);
+msp_status scan_i64_to_i64(const int64_t *in, int64_t *out, int64_t n, void *ws, size_t ws_bytes, cudaStream_t s);
 // In place: counts c[0..n) -> exclusive offsets with c_out[n] = total, int32
 // result; *overflow_dev set to 1 if the total exceeds INT32_MAX.
 msp_status scan_counts_to_offsets_i32(int32_t *counts, int64_t n, int64_t *total_dev, void *ws,

@@ -25,6 +25,10 @@ struct LoadI32 {
     const int32_t *p;
     __device__ int64_t operator()(int64_t i) const { return p[i]; }
 };
+struct LoadI64 {
+    const int64_t *p;
+    __device__ int64_t operator()(int64_t i) const { return p[i]; }
+};
 struct LoadWidth {  // nnz of the B row referenced by A nonzero i
     const int32_t *acol, *brp;
     __device__ int64_t operator()(int64_t i) const
@@ -180,6 +184,11 @@ msp_status scan_counts_to_offsets_i32(int32_t *counts, int64_t n, int64_t *total
     // just before `counts`); int64 accumulation, int32 store
     return run_scan<LoadI32, StoreI32, false>(LoadI32{counts}, StoreI32{counts}, n, total_dev, nullptr, ws,
                                               ws_bytes, s);
+}
+
+msp_status scan_i64_to_i64(const int64_t *in, int64_t *out, int64_t n, void *ws, size_t ws_bytes, cudaStream_t s)
+{
+    return run_scan<LoadI64, StoreI64, true>(LoadI64{in}, StoreI64{out}, n, nullptr, out, ws, ws_bytes, s);
 }
 
 msp_status scan_widths_to_S(const int32_t *Acol, const int32_t *Brp, int64_t nnzA, int64_t *S, void *ws,

@@ -1,0 +1,804 @@
+// spgemm.cu -- C = A B by expansion, sorting and compression (sm_100a).
+//
+// Paper: Section III-C.  Work is measured in products, Nprods
+// (P:888-896).  Setup forms the prefix sum S of the B row lengths referenced
+// by A's column indices (reading Z8: flat int64 exclusive scan);
+// products are split over CTAs with a search over S (reading Z7);
+// every CTA expands its products, sorts them so duplicates become adjacent
+// and reduces them; what straddles CTAs is
+// ordered and reduced in a global phase.
+//
+// B200 design:
+//   * Merge grid = A nonzero ends + products (items), so a tile of T items
+//     holds at most T products and at most T nonzeros whatever the widths.
+//     Tile boundaries are merge-path splits moved to the nearest row
+//     boundary when they fall inside a short row (<= T/4 items), so short
+//     rows never straddle tiles; rows with more than T/4 items ("long rows")
+//     are masked out of the tiles and handled by the global phase.
+//   * Tile kernel (512 threads x 16 products): merge-path expansion from
+//     S (each thread finds its split once, then walks), keys (row, col)
+//     packed in 64 bits, stable block merge sort (sort.cuh), then
+//     compression: symbolic adds each row's unique count into
+//     C.row_offsets; numeric writes each unique (col, sum) at
+//     C.row_offsets[row] + rank of the key in its row (the tile's short
+//     rows are complete).  Duplicates are summed in product order (k
+//     ascending, as Gustavson's oracle), fp64 accumulation (Z4).
+//   * Long rows (global phase): each is cut into chunks of T products, each
+//     chunk expanded and sorted by column into a run; runs are merged pairwise
+//     (merge path per thread, stable) until one run per row remains; a head-
+//     flag pass reduces equal columns (counts, or scan + sums for numeric).
+#include <algorithm>
+#include <climits>
+#include <cstdint>
+#include <cstdio>
+
+#include "common.cuh"
+#include "internal.h"
+#include "sort.cuh"
+
+namespace msp {
+namespace {
+
+constexpr int GM_NT = 512;
+constexpr int GM_IPT = 16;
+constexpr int GM_T = GM_NT * GM_IPT;  // items (nonzero ends + products) per tile
+constexpr int GM_LONG = GM_T / 4;     // rows with more items than this are long
+// Partition step: snapping a split to the nearest short-row boundary moves
+// it by at most GM_LONG / 2, so tiles of GM_TP nominal items never exceed GM_T.
+constexpr int GM_TP = GM_T - GM_LONG;
+constexpr int GM_TL = GM_T;           // products per long-row chunk
+constexpr uint64_t KEY_MASKED = ~0ull;
+constexpr uint64_t KEY_NONE = 1ull << 63;  // never equal to a real key
+
+__device__ __forceinline__ int64_t dmin(int64_t a, int64_t b) { return a < b ? a : b; }
+__device__ __forceinline__ int64_t dmax(int64_t a, int64_t b) { return a > b ? a : b; }
+
+// ================================================================ setup ===
+
+// COO row of every A nonzero, merge-based (equal rows + nonzeros per thread).
+constexpr int AROW_ITEMS = 16;
+__global__ void arow_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, int32_t *__restrict__ arow)
+{
+    const int64_t total = int64_t(m) + nnz;
+    const int64_t d = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) * AROW_ITEMS;
+    if (d >= total) return;
+    int64_t lo = dmax(0, d - nnz), hi = dmin(d, m);
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (int64_t(rp[mid + 1]) <= d - mid - 1) lo = mid + 1;
+        else hi = mid;
+    }
+    int64_t i = lo, j = d - lo;
+    const int64_t end = dmin(d + AROW_ITEMS, total);
+    for (int64_t q = d; q < end; ++q) {
+        if (i < m && rp[i + 1] <= j) ++i;  // row end
+        else arow[j++] = int32_t(i);
+    }
+}
+
+// Per row: products P_r = S[rp[r+1]] - S[rp[r]]; long iff nnz_r + P_r > GM_LONG.
+__global__ void rowclass_kernel(int32_t m, const int32_t *__restrict__ rp, const int64_t *__restrict__ S,
+                                uint8_t *__restrict__ rowlong, int32_t *__restrict__ longflag,
+                                int64_t *__restrict__ longP, unsigned long long *__restrict__ maxP)
+{
+    unsigned long long mx = 0;
+    for (int64_t r = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; r < m; r += int64_t(gridDim.x) * blockDim.x) {
+        const int32_t a = rp[r], b = rp[r + 1];
+        const int64_t P = S[b] - S[a];
+        const bool lg = (int64_t(b - a) + P) > GM_LONG;
+        rowlong[r] = lg ? 1 : 0;
+        longflag[r] = lg ? 1 : 0;
+        longP[r] = 0;
+        mx = max(mx, (unsigned long long)P);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    if ((threadIdx.x & 31) == 0 && mx) atomicMax(maxP, mx);
+}
+
+__global__ void long_scatter_kernel(int32_t m, const int32_t *__restrict__ rp, const int64_t *__restrict__ S,
+                                    const int32_t *__restrict__ longflag, const int64_t *__restrict__ longpos,
+                                    int32_t *__restrict__ longrow, int64_t *__restrict__ longP,
+                                    int64_t *__restrict__ longC)
+{
+    for (int64_t r = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; r < m; r += int64_t(gridDim.x) * blockDim.x) {
+        if (!longflag[r]) continue;
+        const int64_t idx = longpos[r];
+        const int64_t P = S[rp[r + 1]] - S[rp[r]];
+        longrow[idx] = int32_t(r);
+        longP[idx] = P;
+        longC[idx] = (P + GM_TL - 1) / GM_TL;
+    }
+}
+
+struct SetupWs {
+    int32_t *arow;
+    int64_t *S;          // [nnzA + 1]
+    uint8_t *rowlong;    // [m]
+    int32_t *longflag;   // [m]
+    int64_t *longpos;    // [m + 1]
+    int32_t *longrow;    // [m]
+    int64_t *longP;      // [m]  (products of the i-th long row)
+    int64_t *longO;      // [m + 1] prefix of longP
+    int64_t *longC;      // [m]  chunks of the i-th long row
+    int64_t *longCO;     // [m + 1] prefix of longC
+    unsigned long long *stats;  // [4]: max row products
+    void *scan;
+    size_t scan_bytes;
+    size_t bytes;
+};
+
+SetupWs carve_setup(const msp_csr *A, void *ws, size_t cap, bool *ok)
+{
+    SetupWs w;
+    const int64_t m = A->nrows, nnz = A->nnz;
+    Carve cv(ws, cap);
+    w.arow = cv.take<int32_t>(size_t(nnz > 0 ? nnz : 1));
+    w.S = cv.take<int64_t>(size_t(nnz + 1));
+    w.rowlong = cv.take<uint8_t>(size_t(m > 0 ? m : 1));
+    w.longflag = cv.take<int32_t>(size_t(m > 0 ? m : 1));
+    w.longpos = cv.take<int64_t>(size_t(m + 1));
+    w.longrow = cv.take<int32_t>(size_t(m > 0 ? m : 1));
+    w.longP = cv.take<int64_t>(size_t(m > 0 ? m : 1));
+    w.longO = cv.take<int64_t>(size_t(m + 1));
+    w.longC = cv.take<int64_t>(size_t(m > 0 ? m : 1));
+    w.longCO = cv.take<int64_t>(size_t(m + 1));
+    w.stats = cv.take<unsigned long long>(4);
+    w.scan_bytes = scan_ws_bytes(std::max<int64_t>(std::max<int64_t>(m, nnz), 1));
+    w.scan = cv.take<char>(w.scan_bytes);
+    w.bytes = cv.off;
+    *ok = cv.ok();
+    return w;
+}
+
+// ================================================================ main ====
+
+struct GSplit {
+    int64_t j, p;  // nonzero ends consumed, products consumed
+};
+
+__global__ void gemm_partition_kernel(int32_t m, int64_t nnzA, int64_t nprods, const int32_t *__restrict__ Arp,
+                                      const int32_t *__restrict__ arow, const int64_t *__restrict__ S,
+                                      const uint8_t *__restrict__ rowlong, int64_t ntiles, GSplit *__restrict__ splits)
+{
+    const int64_t total = nnzA + nprods;
+    for (int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; k <= ntiles; k += int64_t(gridDim.x) * blockDim.x) {
+        const int64_t d = dmin(k * GM_TP, total);
+        int64_t lo = dmax(0, d - nprods), hi = dmin(d, nnzA);
+        while (lo < hi) {
+            const int64_t mid = (lo + hi) >> 1;
+            if (S[mid + 1] <= d - mid - 1) lo = mid + 1;
+            else hi = mid;
+        }
+        GSplit s{lo, d - lo};
+        if (lo < nnzA && d < total) {
+            // snap to the nearest boundary of a short row (short rows never straddle)
+            const int32_t r = arow[lo];
+            if (!rowlong[r]) {
+                const int64_t j_a = Arp[r], j_b = Arp[r + 1];
+                const int64_t i_a = j_a + S[j_a], i_b = j_b + S[j_b];
+                if (d > i_a && d < i_b) s = (d - i_a <= i_b - d) ? GSplit{j_a, S[j_a]} : GSplit{j_b, S[j_b]};
+            }
+        }
+        splits[k] = s;
+    }
+}
+
+template <typename V, bool NUM>
+struct TileSmem {
+    BlockSortSmem<GM_NT, GM_IPT> sort;  // sort.keys doubles as the expansion staging buffer
+    double vals[NUM ? GM_T : 1];
+    uint64_t edge_first[GM_NT];
+    uint64_t edge_last[GM_NT];
+    SegPair<double> scan_w[GM_NT / 32];
+    int32_t wsum[GM_NT / 32];
+};
+
+// One CTA per tile: expand -> sort by (row, col) -> compress.
+template <typename V, bool NUM>
+__global__ void __launch_bounds__(GM_NT)
+gemm_tile_kernel(const int32_t *__restrict__ Acol, const V *__restrict__ Aval, const int32_t *__restrict__ Brp,
+                 const int32_t *__restrict__ Bcol, const V *__restrict__ Bval, const int32_t *__restrict__ arow,
+                 const int64_t *__restrict__ S, const uint8_t *__restrict__ rowlong, const GSplit *__restrict__ splits,
+                 int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol, V *__restrict__ Cval)
+{
+    extern __shared__ __align__(16) char smem_raw[];
+    TileSmem<V, NUM> &Sm = *reinterpret_cast<TileSmem<V, NUM> *>(smem_raw);
+    const int tid = threadIdx.x;
+    const GSplit s0 = splits[blockIdx.x], s1 = splits[blockIdx.x + 1];
+    const int64_t j0 = s0.j, p0 = s0.p;
+    const int nz = int(s1.j - j0), np = int(s1.p - p0);
+    if (np == 0) return;
+    const int32_t rbase = arow[j0];
+    // ---- expansion: merge path over (nonzero ends, products) of the tile ----
+    {
+        const int items = nz + np;
+        const int dt = min(tid * GM_IPT, items);
+        int lo = max(0, dt - np), hi = min(dt, nz);
+        while (lo < hi) {
+            const int mid = (lo + hi) >> 1;
+            if (S[j0 + mid + 1] - p0 <= dt - mid - 1) lo = mid + 1;
+            else hi = mid;
+        }
+        int64_t j = j0 + lo;
+        int64_t p = p0 + (dt - lo);
+        const int64_t jend = j0 + nz;
+        const int todo = min(GM_IPT, items - dt);
+        int64_t sj1 = (j < jend) ? S[j + 1] : INT64_MAX;
+        int64_t bofs = 0;
+        uint64_t rowkey = 0;
+        bool masked = true;
+        double av = 0.0;
+        bool loaded = false;
+        for (int q = 0; q < todo; ++q) {
+            if (j < jend && sj1 <= p) {  // nonzero j ends
+                ++j;
+                sj1 = (j < jend) ? S[j + 1] : INT64_MAX;
+                loaded = false;
+                continue;
+            }
+            if (!loaded) {
+                const int32_t r = arow[j];
+                masked = rowlong[r] != 0;
+                rowkey = uint64_t(uint32_t(r - rbase)) << 32;
+                const int32_t kk = Acol[j];
+                bofs = int64_t(Brp[kk]) - S[j];
+                if (NUM) av = double(Aval[j]);
+                loaded = true;
+            }
+            const int slot = int(p - p0);
+            const int64_t bi = bofs + p;
+            Sm.sort.keys[slot] = masked ? KEY_MASKED : (rowkey | uint32_t(Bcol[bi]));
+            if (NUM) Sm.vals[slot] = av * double(Bval[bi]);
+            ++p;
+        }
+    }
+    __syncthreads();
+    // ---- sort the tile's products by (row, col), stable ----
+    uint64_t k[GM_IPT];
+    int v[GM_IPT];
+#pragma unroll
+    for (int u = 0; u < GM_IPT; ++u) {
+        const int slot = tid + u * GM_NT;
+        k[u] = slot < np ? Sm.sort.keys[slot] : KEY_MASKED;
+        v[u] = slot;
+    }
+    __syncthreads();  // staging is reused by the sort
+    block_merge_sort<GM_NT, GM_IPT>(k, v, Sm.sort);
+    // neighbours across thread boundaries
+    Sm.edge_first[tid] = k[0];
+    Sm.edge_last[tid] = k[GM_IPT - 1];
+    __syncthreads();
+    const uint64_t prevk = tid > 0 ? Sm.edge_last[tid - 1] : KEY_NONE;
+    const uint64_t nextk = tid + 1 < GM_NT ? Sm.edge_first[tid + 1] : KEY_NONE;
+
+    if (!NUM) {
+        // ---- unique count per row (rows are complete in the tile) ----
+        uint64_t pk = prevk;
+        int cnt = 0;
+        int64_t row = -1;
+#pragma unroll
+        for (int i = 0; i < GM_IPT; ++i) {
+            if (k[i] != KEY_MASKED) {
+                const int64_t r = int64_t(rbase) + int64_t(k[i] >> 32);
+                if (r != row) {
+                    if (cnt) atomicAdd(&Crp[row + 1], cnt);
+                    cnt = 0;
+                    row = r;
+                }
+                if (k[i] != pk) ++cnt;
+            }
+            pk = k[i];
+        }
+        if (cnt) atomicAdd(&Crp[row + 1], cnt);
+    } else {
+        // ---- unique (col, sum): position = C.rp[row] + rank of the key in its row ----
+        int heads = 0, last_rs = -1;  // heads in this thread; heads before its last row start
+        double trail = 0.0;           // sum after the last head in this thread
+        {
+            uint64_t pk = prevk;
+#pragma unroll
+            for (int i = 0; i < GM_IPT; ++i) {
+                if (k[i] != KEY_MASKED) {
+                    const double val = Sm.vals[v[i]];
+                    if (k[i] != pk) {
+                        if (pk == KEY_MASKED || pk == KEY_NONE || (pk >> 32) != (k[i] >> 32)) last_rs = heads;
+                        ++heads;
+                        trail = val;
+                    } else {
+                        trail = trail + val;
+                    }
+                }
+                pk = k[i];
+            }
+        }
+        int tot;
+        const int u0 = block_exclusive_sum<int, GM_NT / 32>(heads, Sm.wsum, 0, &tot);
+        SegPair<double> all;
+        const SegPair<double> carry =
+            block_seg_exclusive<double, GM_NT / 32>(SegPair<double>{heads > 0, trail}, SegPair<double>{0, 0.0},
+                                                    Sm.scan_w, 0, &all);
+        // tile rank of the first key of the row open at this thread's start
+        const int rs_carry = block_exclusive_max<GM_NT / 32>(last_rs >= 0 ? u0 + last_rs : -1, Sm.wsum, 0);
+        uint64_t pk = prevk;
+        int u = u0 - 1, row_u = rs_carry;
+        double run = carry.v;
+#pragma unroll
+        for (int i = 0; i < GM_IPT; ++i) {
+            if (k[i] != KEY_MASKED) {
+                const double val = Sm.vals[v[i]];
+                if (k[i] != pk) {
+                    ++u;
+                    if (pk == KEY_MASKED || pk == KEY_NONE || (pk >> 32) != (k[i] >> 32)) row_u = u;
+                    run = val;
+                } else {
+                    run = run + val;
+                }
+                const uint64_t nk = (i + 1 < GM_IPT) ? k[i + 1] : nextk;
+                if (nk != k[i]) {  // run ends here
+                    const int64_t row = int64_t(rbase) + int64_t(k[i] >> 32);
+                    const int64_t pos = int64_t(Crp[row]) + (u - row_u);
+                    Ccol[pos] = int32_t(uint32_t(k[i]));
+                    Cval[pos] = V(run);
+                }
+            }
+            pk = k[i];
+        }
+    }
+}
+
+// ---------------------------------------------------------- long rows ----
+
+template <typename V, bool NUM>
+struct LongSmem {
+    BlockSortSmem<GM_NT, GM_IPT> sort;
+    double vals[NUM ? GM_TL : 1];
+};
+
+// Chunk c of long row l: expand products [c*TL, ...) of the row, sort by
+// column (stable), write the sorted run at longO[l] + c*TL.
+template <typename V, bool NUM>
+__global__ void __launch_bounds__(GM_NT)
+long_chunk_kernel(const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol, const V *__restrict__ Aval,
+                  const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol, const V *__restrict__ Bval,
+                  const int64_t *__restrict__ S, int64_t nlong, const int32_t *__restrict__ longrow,
+                  const int64_t *__restrict__ longP, const int64_t *__restrict__ longO,
+                  const int64_t *__restrict__ longCO, int32_t *__restrict__ Xcol, double *__restrict__ Xval)
+{
+    extern __shared__ __align__(16) char smem_raw[];
+    LongSmem<V, NUM> &Sm = *reinterpret_cast<LongSmem<V, NUM> *>(smem_raw);
+    const int tid = threadIdx.x;
+    const int64_t b = blockIdx.x;
+    int64_t lo = 0, hi = nlong;  // l: last with longCO[l] <= b
+    while (hi - lo > 1) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (longCO[mid] <= b) lo = mid;
+        else hi = mid;
+    }
+    const int64_t l = lo;
+    const int64_t c = b - longCO[l];
+    const int32_t r = longrow[l];
+    const int64_t P = longP[l];
+    const int64_t q0 = c * GM_TL;
+    const int nq = int(dmin(GM_TL, P - q0));
+    const int64_t ja = Arp[r], jb = Arp[r + 1];
+    const int64_t pr0 = S[ja];  // global product index of the row's first product
+    uint64_t k[GM_IPT];
+    int v[GM_IPT];
+    {
+        const int64_t qs = q0 + int64_t(tid) * GM_IPT;
+        // nonzero of product pr0 + qs: last j in [ja, jb) with S[j] <= pr0 + qs
+        int64_t j = ja;
+        if (qs < P) {
+            int64_t lo2 = ja, hi2 = jb;
+            const int64_t pg = pr0 + qs;
+            while (hi2 - lo2 > 1) {
+                const int64_t mid = (lo2 + hi2) >> 1;
+                if (S[mid] <= pg) lo2 = mid;
+                else hi2 = mid;
+            }
+            j = lo2;
+        }
+        int64_t sj1 = S[j + 1];
+        int64_t bofs = int64_t(Brp[Acol[j]]) - S[j];
+        double av = NUM ? double(Aval[j]) : 0.0;
+#pragma unroll
+        for (int i = 0; i < GM_IPT; ++i) {
+            const int64_t q = qs + i;
+            const int slot = tid * GM_IPT + i;
+            v[i] = slot;
+            if (q < q0 + nq) {
+                const int64_t pg = pr0 + q;
+                while (sj1 <= pg) {  // skip to the nonzero holding product pg
+                    ++j;
+                    sj1 = S[j + 1];
+                    bofs = int64_t(Brp[Acol[j]]) - S[j];
+                    if (NUM) av = double(Aval[j]);
+                }
+                const int64_t bi = bofs + pg;
+                k[i] = uint32_t(Bcol[bi]);
+                if (NUM) Sm.vals[slot] = av * double(Bval[bi]);
+            } else {
+                k[i] = KEY_MASKED;
+            }
+        }
+    }
+    __syncthreads();
+    block_merge_sort<GM_NT, GM_IPT>(k, v, Sm.sort);
+    const int64_t out = longO[l] + q0;
+#pragma unroll
+    for (int i = 0; i < GM_IPT; ++i) {
+        const int pos = tid * GM_IPT + i;
+        if (pos < nq) {
+            Xcol[out + pos] = int32_t(k[i]);
+            if (NUM) Xval[out + pos] = Sm.vals[v[i]];
+        }
+    }
+}
+
+// One merge pass: runs of `w` entries inside each long row are merged
+// pairwise (stable, left run first).  Each thread produces 16 outputs.
+template <bool NUM>
+__global__ void long_merge_kernel(int64_t LP, int64_t nlong, const int64_t *__restrict__ longO,
+                                  const int64_t *__restrict__ longP, int64_t w, const int32_t *__restrict__ Xc,
+                                  const double *__restrict__ Xv, int32_t *__restrict__ Yc, double *__restrict__ Yv)
+{
+    int64_t e = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) * 16;
+    const int64_t e_end = dmin(e + 16, LP);
+    while (e < e_end) {
+        int64_t lo = 0, hi = nlong;
+        while (hi - lo > 1) {
+            const int64_t mid = (lo + hi) >> 1;
+            if (longO[mid] <= e) lo = mid;
+            else hi = mid;
+        }
+        const int64_t O = longO[lo], P = longP[lo];
+        const int64_t q = e - O;
+        const int64_t a0 = (q / (2 * w)) * (2 * w);
+        const int64_t la = dmin(w, P - a0);
+        const int64_t lb = dmax(0, dmin(w, P - a0 - la));
+        const int64_t d = q - a0;
+        const int64_t A0 = O + a0, B0 = O + a0 + la;
+        int64_t l2 = dmax(0, d - lb), h2 = dmin(d, la);
+        while (l2 < h2) {
+            const int64_t mid = (l2 + h2) >> 1;
+            if (Xc[A0 + mid] <= Xc[B0 + d - mid - 1]) l2 = mid + 1;
+            else h2 = mid;
+        }
+        int64_t ia = l2, ib = d - l2;
+        const int64_t n = dmin(e_end - e, la + lb - d);
+        for (int64_t t = 0; t < n; ++t) {
+            const bool ta = ib >= lb || (ia < la && Xc[A0 + ia] <= Xc[B0 + ib]);
+            if (ta) {
+                Yc[e + t] = Xc[A0 + ia];
+                if (NUM) Yv[e + t] = Xv[A0 + ia];
+                ++ia;
+            } else {
+                Yc[e + t] = Xc[B0 + ib];
+                if (NUM) Yv[e + t] = Xv[B0 + ib];
+                ++ib;
+            }
+        }
+        e += n;
+    }
+}
+
+// Head flags of the sorted long rows; symbolic adds per-row unique counts.
+__global__ void long_heads_kernel(int64_t LP, int64_t nlong, const int64_t *__restrict__ longO,
+                                  const int32_t *__restrict__ longrow, const int32_t *__restrict__ Fc,
+                                  int32_t *__restrict__ heads, int32_t *__restrict__ Crp_counts)
+{
+    const int64_t e0 = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) * 16;
+    if (e0 >= LP) return;
+    int64_t lo = 0, hi = nlong;
+    while (hi - lo > 1) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (longO[mid] <= e0) lo = mid;
+        else hi = mid;
+    }
+    int64_t l = lo;
+    int64_t rowend = (l + 1 < nlong) ? longO[l + 1] : LP;
+    int cnt = 0;
+    const int64_t e1 = dmin(e0 + 16, LP);
+    for (int64_t e = e0; e < e1; ++e) {
+        while (e >= rowend) {
+            if (cnt && Crp_counts) atomicAdd(&Crp_counts[longrow[l]], cnt);
+            cnt = 0;
+            ++l;
+            rowend = (l + 1 < nlong) ? longO[l + 1] : LP;
+        }
+        const int h = (e == longO[l] || Fc[e] != Fc[e - 1]) ? 1 : 0;
+        if (heads) heads[e] = h;
+        cnt += h;
+    }
+    if (cnt && Crp_counts) atomicAdd(&Crp_counts[longrow[l]], cnt);
+}
+
+// Numeric: every head writes (col, sum of its run) at C.rp[row] + rank.
+template <typename V>
+__global__ void long_emit_kernel(int64_t LP, int64_t nlong, const int64_t *__restrict__ longO,
+                                 const int32_t *__restrict__ longrow, const int32_t *__restrict__ Fc,
+                                 const double *__restrict__ Fv, const int32_t *__restrict__ heads,
+                                 const int64_t *__restrict__ U, const int32_t *__restrict__ Crp,
+                                 int32_t *__restrict__ Ccol, V *__restrict__ Cval)
+{
+    for (int64_t e = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; e < LP; e += int64_t(gridDim.x) * blockDim.x) {
+        if (!heads[e]) continue;
+        int64_t lo = 0, hi = nlong;
+        while (hi - lo > 1) {
+            const int64_t mid = (lo + hi) >> 1;
+            if (longO[mid] <= e) lo = mid;
+            else hi = mid;
+        }
+        const int64_t O = longO[lo];
+        const int64_t rowend = (lo + 1 < nlong) ? longO[lo + 1] : LP;
+        const int64_t pos = int64_t(Crp[longrow[lo]]) + (U[e] - U[O]);
+        double s = Fv[e];
+        for (int64_t e2 = e + 1; e2 < rowend && !heads[e2]; ++e2) s = s + Fv[e2];
+        Ccol[pos] = Fc[e];
+        Cval[pos] = V(s);
+    }
+}
+
+struct MainWs {
+    GSplit *splits;
+    int32_t *Xc[2];
+    double *Xv[2];
+    int32_t *heads;
+    int64_t *U;
+    int64_t *totals;
+    void *scan;
+    size_t scan_bytes;
+    size_t bytes;
+};
+
+MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, void *ws, size_t cap, bool *ok)
+{
+    MainWs w;
+    Carve cv(ws, cap);
+    w.splits = cv.take<GSplit>(size_t(ntiles + 1));
+    for (int i = 0; i < 2; ++i) {
+        w.Xc[i] = cv.take<int32_t>(size_t(LP > 0 ? LP : 1));
+        w.Xv[i] = cv.take<double>(size_t(LP > 0 ? LP : 1));
+    }
+    w.heads = cv.take<int32_t>(size_t(LP > 0 ? LP : 1));
+    w.U = cv.take<int64_t>(size_t(LP + 1));
+    w.totals = cv.take<int64_t>(4);
+    w.scan_bytes = scan_ws_bytes(std::max<int64_t>(std::max<int64_t>(m, LP), 1));
+    w.scan = cv.take<char>(w.scan_bytes);
+    w.bytes = cv.off;
+    *ok = cv.ok();
+    return w;
+}
+
+struct HostInfo {  // read back by setup, re-derived by symbolic / numeric
+    int64_t nprods, nlong, LP, LC, maxP;
+};
+
+msp_status read_info(const SetupWs &sw, int64_t m, int64_t nnzA, HostInfo *h, cudaStream_t s)
+{
+    int64_t v[5] = {0, 0, 0, 0, 0};
+    msp_status st = cuda_check(cudaMemcpyAsync(&v[0], &sw.S[nnzA], 8, cudaMemcpyDeviceToHost, s), "spgemm: info");
+    if (st == MSP_OK) st = cuda_check(cudaMemcpyAsync(&v[1], &sw.longpos[m], 8, cudaMemcpyDeviceToHost, s), "info");
+    if (st == MSP_OK) st = cuda_check(cudaMemcpyAsync(&v[4], sw.stats, 8, cudaMemcpyDeviceToHost, s), "info");
+    if (st == MSP_OK) st = cuda_check(cudaStreamSynchronize(s), "spgemm: sync");
+    if (st != MSP_OK) return st;
+    h->nprods = v[0];
+    h->nlong = v[1];
+    h->maxP = v[4];
+    if (h->nlong > 0) {
+        st = cuda_check(cudaMemcpyAsync(&v[2], &sw.longO[h->nlong], 8, cudaMemcpyDeviceToHost, s), "info");
+        if (st == MSP_OK) st = cuda_check(cudaMemcpyAsync(&v[3], &sw.longCO[h->nlong], 8, cudaMemcpyDeviceToHost, s), "info");
+        if (st == MSP_OK) st = cuda_check(cudaStreamSynchronize(s), "spgemm: sync");
+        if (st != MSP_OK) return st;
+    }
+    h->LP = v[2];
+    h->LC = v[3];
+    return MSP_OK;
+}
+
+template <typename V, bool NUM>
+msp_status run_tiles(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, int64_t ntiles,
+                     int32_t *Crp, int32_t *Ccol, void *Cval, cudaStream_t s)
+{
+    auto kern = gemm_tile_kernel<V, NUM>;
+    const int smem = int(sizeof(TileSmem<V, NUM>));
+    static int configured = 0;
+    if (!configured) {
+        msp_status st = cuda_check(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem),
+                                   "spgemm: tile smem");
+        if (st != MSP_OK) return st;
+        configured = 1;
+    }
+    if (ntiles <= 0) return MSP_OK;
+    kern<<<unsigned(ntiles), GM_NT, smem, s>>>(A->col_idx, static_cast<const V *>(A->vals), B->row_offsets,
+                                                B->col_idx, static_cast<const V *>(B->vals), sw.arow, sw.S,
+                                                sw.rowlong, mw.splits, Crp, Ccol, static_cast<V *>(Cval));
+    return last_launch("gemm_tile_kernel");
+}
+
+template <typename V, bool NUM>
+msp_status run_long(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, const HostInfo &h,
+                    int32_t *Crp, int32_t *Ccol, void *Cval, cudaStream_t s)
+{
+    if (h.nlong == 0 || h.LP == 0) return MSP_OK;
+    auto ck = long_chunk_kernel<V, NUM>;
+    const int smem = int(sizeof(LongSmem<V, NUM>));
+    static int configured = 0;
+    if (!configured) {
+        msp_status st = cuda_check(cudaFuncSetAttribute(ck, cudaFuncAttributeMaxDynamicSharedMemorySize, smem),
+                                   "spgemm: chunk smem");
+        if (st != MSP_OK) return st;
+        configured = 1;
+    }
+    ck<<<unsigned(h.LC), GM_NT, smem, s>>>(A->row_offsets, A->col_idx, static_cast<const V *>(A->vals),
+                                           B->row_offsets, B->col_idx, static_cast<const V *>(B->vals), sw.S,
+                                           h.nlong, sw.longrow, sw.longP, sw.longO, sw.longCO, mw.Xc[0], mw.Xv[0]);
+    msp_status st = last_launch("long_chunk_kernel");
+    if (st != MSP_OK) return st;
+    int cur = 0;
+    int64_t maxlong = h.maxP;
+    for (int64_t w = GM_TL; w < maxlong; w *= 2) {
+        const int64_t threads = ceil_div(h.LP, 16);
+        long_merge_kernel<NUM><<<unsigned(ceil_div(threads, 256)), 256, 0, s>>>(
+            h.LP, h.nlong, sw.longO, sw.longP, w, mw.Xc[cur], mw.Xv[cur], mw.Xc[cur ^ 1], mw.Xv[cur ^ 1]);
+        st = last_launch("long_merge_kernel");
+        if (st != MSP_OK) return st;
+        cur ^= 1;
+    }
+    const unsigned hb = unsigned(ceil_div(ceil_div(h.LP, 16), 256));
+    if (!NUM) {
+        long_heads_kernel<<<hb, 256, 0, s>>>(h.LP, h.nlong, sw.longO, sw.longrow, mw.Xc[cur], nullptr, Crp + 1);
+        return last_launch("long_heads_kernel");
+    }
+    long_heads_kernel<<<hb, 256, 0, s>>>(h.LP, h.nlong, sw.longO, sw.longrow, mw.Xc[cur], mw.heads, nullptr);
+    st = last_launch("long_heads_kernel");
+    if (st != MSP_OK) return st;
+    st = scan_i32_to_i64(mw.heads, mw.U, h.LP, mw.scan, mw.scan_bytes, s);
+    if (st != MSP_OK) return st;
+    const unsigned eb = unsigned(std::min<int64_t>(ceil_div(h.LP, 256), 148 * 16));
+    long_emit_kernel<V><<<eb, 256, 0, s>>>(h.LP, h.nlong, sw.longO, sw.longrow, mw.Xc[cur], mw.Xv[cur], mw.heads,
+                                           mw.U, Crp, Ccol, static_cast<V *>(Cval));
+    return last_launch("long_emit_kernel");
+}
+
+int64_t ntiles_of(int64_t nnzA, int64_t nprods) { return ceil_div(nnzA + nprods > 0 ? nnzA + nprods : 1, GM_TP); }
+
+msp_status prepare_main(const msp_csr *A, const void *ws1, size_t b1, void *ws2, size_t b2, SetupWs *sw, MainWs *mw,
+                        HostInfo *h, cudaStream_t s)
+{
+    bool ok1, ok2;
+    *sw = carve_setup(A, const_cast<void *>(ws1), b1, &ok1);
+    if (!ok1) return MSP_ERR_WORKSPACE;
+    msp_status st = read_info(*sw, A->nrows, A->nnz, h, s);
+    if (st != MSP_OK) return st;
+    *mw = carve_main(A->nrows, ntiles_of(A->nnz, h->nprods), h->LP, ws2, b2, &ok2);
+    if (!ok2) return MSP_ERR_WORKSPACE;
+    return MSP_OK;
+}
+
+}  // namespace
+
+size_t spgemm_setup_ws_bytes(const msp_csr *A, const msp_csr *)
+{
+    bool ok;
+    SetupWs w = carve_setup(A, nullptr, SIZE_MAX, &ok);
+    return w.bytes + 256;
+}
+
+msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_t b1, msp_spgemm_info *info,
+                            cudaStream_t s)
+{
+    bool ok;
+    SetupWs w = carve_setup(A, ws1, b1, &ok);
+    if (!ok) return MSP_ERR_WORKSPACE;
+    const int64_t m = A->nrows, nnz = A->nnz;
+    msp_status st = cuda_check(cudaMemsetAsync(w.stats, 0, 4 * sizeof(unsigned long long), s), "spgemm: clear");
+    if (st != MSP_OK) return st;
+    if (nnz > 0) {
+        const int64_t thr = ceil_div(m + nnz, AROW_ITEMS);
+        arow_kernel<<<unsigned(ceil_div(thr, 256)), 256, 0, s>>>(A->nrows, nnz, A->row_offsets, w.arow);
+        st = last_launch("arow_kernel");
+        if (st != MSP_OK) return st;
+    }
+    st = scan_widths_to_S(A->col_idx, B->row_offsets, nnz, w.S, w.scan, w.scan_bytes, s);
+    if (st != MSP_OK) return st;
+    if (m > 0) {
+        const unsigned blocks = unsigned(std::min<int64_t>(ceil_div(m, 256), 148 * 16));
+        rowclass_kernel<<<blocks, 256, 0, s>>>(A->nrows, A->row_offsets, w.S, w.rowlong, w.longflag, w.longP,
+                                               w.stats);
+        st = last_launch("rowclass_kernel");
+        if (st != MSP_OK) return st;
+        st = scan_i32_to_i64(w.longflag, w.longpos, m, w.scan, w.scan_bytes, s);
+        if (st != MSP_OK) return st;
+        st = cuda_check(cudaMemsetAsync(w.longC, 0, size_t(m) * sizeof(int64_t), s), "spgemm: clear");
+        if (st != MSP_OK) return st;
+        long_scatter_kernel<<<blocks, 256, 0, s>>>(A->nrows, A->row_offsets, w.S, w.longflag, w.longpos,
+                                                   w.longrow, w.longP, w.longC);
+        st = last_launch("long_scatter_kernel");
+        if (st != MSP_OK) return st;
+        st = scan_i64_to_i64(w.longP, w.longO, m, w.scan, w.scan_bytes, s);
+        if (st != MSP_OK) return st;
+        st = scan_i64_to_i64(w.longC, w.longCO, m, w.scan, w.scan_bytes, s);
+        if (st != MSP_OK) return st;
+    } else {
+        st = cuda_check(cudaMemsetAsync(w.longpos, 0, sizeof(int64_t), s), "spgemm: clear");
+        if (st != MSP_OK) return st;
+    }
+    HostInfo h;
+    st = read_info(w, m, nnz, &h, s);
+    if (st != MSP_OK) return st;
+    const int64_t ntiles = ntiles_of(nnz, h.nprods);
+    bool ok2;
+    MainWs mw = carve_main(m, ntiles, h.LP, nullptr, SIZE_MAX, &ok2);
+    info->nprods = h.nprods;
+    info->ntiles = ntiles;
+    info->long_rows = h.nlong;
+    info->long_products = h.LP;
+    info->max_row_products = h.maxP;
+    info->main_ws_bytes = int64_t(mw.bytes + 256);
+    return MSP_OK;
+}
+
+template <bool NUM>
+msp_status spgemm_pass(const msp_csr *A, const msp_csr *B, const void *ws1, size_t b1, void *ws2, size_t b2,
+                       int32_t *Crp, int32_t *Ccol, void *Cval, int64_t *nnzC, cudaStream_t s)
+{
+    SetupWs sw;
+    MainWs mw;
+    HostInfo h;
+    msp_status st = prepare_main(A, ws1, b1, ws2, b2, &sw, &mw, &h, s);
+    if (st != MSP_OK) return st;
+    const int64_t m = A->nrows;
+    const int64_t ntiles = ntiles_of(A->nnz, h.nprods);
+    if (!NUM) {
+        st = cuda_check(cudaMemsetAsync(Crp, 0, size_t(m + 1) * sizeof(int32_t), s), "spgemm: clear rp");
+        if (st != MSP_OK) return st;
+        if (m == 0) {
+            *nnzC = 0;
+            return cuda_check(cudaStreamSynchronize(s), "spgemm: sync");
+        }
+        gemm_partition_kernel<<<unsigned(std::min<int64_t>(ceil_div(ntiles + 1, 256), 148 * 16)), 256, 0, s>>>(
+            A->nrows, A->nnz, h.nprods, A->row_offsets, sw.arow, sw.S, sw.rowlong, ntiles, mw.splits);
+        st = last_launch("gemm_partition_kernel");
+        if (st != MSP_OK) return st;
+    } else if (m == 0 || h.nprods == 0) {
+        return MSP_OK;
+    }
+    if (h.nprods > 0) {
+        st = (A->dtype == MSP_F64) ? run_tiles<double, NUM>(A, B, sw, mw, ntiles, Crp, Ccol, Cval, s)
+                                   : run_tiles<float, NUM>(A, B, sw, mw, ntiles, Crp, Ccol, Cval, s);
+        if (st != MSP_OK) return st;
+        st = (A->dtype == MSP_F64) ? run_long<double, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s)
+                                   : run_long<float, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s);
+        if (st != MSP_OK) return st;
+    }
+    if (!NUM) {
+        st = scan_counts_to_offsets_i32(Crp + 1, m, &mw.totals[0], mw.scan, mw.scan_bytes, s);
+        if (st != MSP_OK) return st;
+        int64_t tot = 0;
+        st = cuda_check(cudaMemcpyAsync(&tot, &mw.totals[0], 8, cudaMemcpyDeviceToHost, s), "spgemm: nnz");
+        if (st == MSP_OK) st = cuda_check(cudaStreamSynchronize(s), "spgemm: sync");
+        if (st != MSP_OK) return st;
+        *nnzC = tot;
+        if (tot > INT32_MAX) {
+            set_error("spgemm: nnz(C) = %lld exceeds int32", (long long)tot);
+            return MSP_ERR_OVERFLOW;
+        }
+    }
+    return MSP_OK;
+}
+
+msp_status spgemm_symbolic_run(const msp_csr *A, const msp_csr *B, const void *ws1, size_t b1, void *ws2,
+                               size_t b2, int32_t *Crp, int64_t *nnzC, cudaStream_t s)
+{
+    return spgemm_pass<false>(A, B, ws1, b1, ws2, b2, Crp, nullptr, nullptr, nnzC, s);
+}
+
+msp_status spgemm_numeric_run(const msp_csr *A, const msp_csr *B, const void *ws1, size_t b1, void *ws2,
+                              size_t b2, const int32_t *Crp, int32_t *Ccol, void *Cval, cudaStream_t s)
+{
+    return spgemm_pass<true>(A, B, ws1, b1, ws2, b2, const_cast<int32_t *>(Crp), Ccol, Cval, nullptr, s);
+}
+
+}  // namespace msp
