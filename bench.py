@@ -228,7 +228,6 @@ def msp_arm(args):
 
     stream = torch.cuda.current_stream(dev)
     ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
-    launches = {"spmv": 1, "spadd": 0, "spgemm": 0}
     rec = {k: [] for k in ("spmv", "allgather", "spadd", "spgemm", "step")}
     extra = {}
 
@@ -285,6 +284,8 @@ def msp_arm(args):
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize(dev)
+    L = msp.lib()
+    n_launch0 = L.msp_launch_count()
     t_start = ev(); t_end = ev()
     t_start.record(stream)
     for _ in range(args.steps):
@@ -294,6 +295,7 @@ def msp_arm(args):
     if world > 1:
         dist.barrier()
     clocks = clk.stop()
+    n_launches = int(L.msp_launch_count() - n_launch0)
     total_ms = t_start.elapsed_time(t_end)
 
     def red_max(v):
@@ -346,7 +348,7 @@ def msp_arm(args):
                          "peak_kind": peak_kind, "unit": "GB/s", "frac": achieved / peak,
                          "alg_bytes_per_launch": by_loc, "traffic": None},
             "clocks": clocks,
-            "gpu_launches": launches["spmv"] * args.spmv_reps * args.steps,
+            "gpu_launches": n_launches,
             "e2e": e2e,
             "cpu_baseline": cpu,
         }

@@ -1,7 +1,8 @@
 """Build libmsp.so in-tree with nvcc for sm_100a (no JIT, no torch extension).
 
-``python -m paper_conf_ipps_daltonbmog15_b200._build`` or
-``__graft_entry__.build()``.  Objects are compiled in parallel and linked
+``python paper_conf_ipps_daltonbmog15_b200/_build.py`` or
+``__graft_entry__.build()`` (run it by path: importing the package loads
+libmsp.so first).  Objects are compiled in parallel and linked
 into ``paper_conf_ipps_daltonbmog15_b200/libmsp.so`` with static cudart and a
 version script that exports only the ``msp_*`` C ABI of include/msp.h.
 """

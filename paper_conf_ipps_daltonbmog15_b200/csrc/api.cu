@@ -6,6 +6,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <atomic>
 #include <mutex>
 
 #include "internal.h"
@@ -31,7 +32,15 @@ msp_status cuda_check(cudaError_t e, const char *where)
     return MSP_ERR_CUDA;
 }
 
-msp_status last_launch(const char *where) { return cuda_check(cudaGetLastError(), where); }
+static std::atomic<uint64_t> g_launches{0};
+
+msp_status last_launch(const char *where)
+{
+    g_launches.fetch_add(1, std::memory_order_relaxed);
+    return cuda_check(cudaGetLastError(), where);
+}
+
+uint64_t launch_count() { return g_launches.load(std::memory_order_relaxed); }
 
 int sm_count()
 {
@@ -104,6 +113,8 @@ const char *msp_status_string(int status)
 const char *msp_last_error(void) { return g_err; }
 
 int msp_version(void) { return MSP_VERSION; }
+
+uint64_t msp_launch_count(void) { return launch_count(); }
 
 // ------------------------------------------------------------------ SpMV
 msp_status msp_spmv_workspace(const msp_csr *A, size_t *bytes)

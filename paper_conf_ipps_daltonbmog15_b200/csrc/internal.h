@@ -18,7 +18,8 @@ int sm_count();
 
 // returns MSP_OK or MSP_ERR_CUDA with the error text recorded
 msp_status cuda_check(cudaError_t e, const char *where);
-msp_status last_launch(const char *where);
+msp_status last_launch(const char *where);  // also counts the launch
+uint64_t launch_count();
 
 inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
