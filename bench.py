@@ -196,11 +196,7 @@ def msp_arm(args):
     xg = gen.x_vector(G.n, "random", seed=1002)
     x_full = torch.as_tensor(xg, device=dev)
     # x slice owned by this rank (equal slices, padded) for the all-gather
-    nsl = -(-G.n // world)
-    x_pad = torch.zeros(nsl * world, dtype=torch.float64, device=dev)
-    x_pad[:G.n] = x_full
-    x_slice = x_pad[rank * nsl:(rank + 1) * nsl].clone()
-    x_gath = torch.empty_like(x_pad)
+    x_slice = msp.dist.x_slice_of(x_full, rank, world)
     y = torch.empty(m_loc, dtype=torch.float64, device=dev)
 
     have = {"spmv": True, "spadd": "spadd" in ops, "spgemm": "spgemm" in ops}
@@ -218,7 +214,7 @@ def msp_arm(args):
                 raise
             have["spadd"] = False
     if have["spgemm"]:
-        Bfull = msp.CsrTensor.from_arrays(G.rp, G.col, G.val, (G.m, G.n), dev) if world > 1 else A
+        Bfull = msp.dist.gather_csr_blocks(A) if world > 1 else A
         try:
             msp.SpGemmPlan(A, Bfull).setup()
         except msp.MspError as e:
@@ -236,9 +232,8 @@ def msp_arm(args):
         # SpMV (x all-gathered over NCCL when distributed)
         if world > 1:
             ea = ev(); ea.record(stream)
-            dist.all_gather_into_tensor(x_gath, x_slice)
+            xin = msp.dist.allgather_x(x_slice, G.n)  # NCCL all-gather of x over NVLink
             eb = ev(); eb.record(stream)
-            xin = x_gath[:G.n]
         else:
             xin = x_full
         sp_ev = []
@@ -256,7 +251,9 @@ def msp_arm(args):
             extra["spadd_nnz_c"] = C.nnz
         if have["spgemm"]:
             g0 = ev(); g0.record(stream)
-            P = msp.SpGemmPlan(A, Bfull)
+            # multi-GPU: replicate B's row blocks (the SpGEMM exchange step)
+            Bg = msp.dist.gather_csr_blocks(A) if world > 1 else Bfull
+            P = msp.SpGemmPlan(A, Bg)
             P.setup()
             P.symbolic()
             Cg = P.numeric()

@@ -8,4 +8,6 @@ from ._lib import EXPORTS, MspError, lib  # noqa: F401
 from .ops import (CsrTensor, SpAddPlan, SpGemmPlan, csr_check, rebase_offsets, row_split,  # noqa: F401
                   spadd, spgemm, spmv, spmv_workspace_bytes, workspace)
 
+from . import dist  # noqa: F401,E402
+
 lib()
