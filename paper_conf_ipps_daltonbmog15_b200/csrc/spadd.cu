@@ -109,10 +109,6 @@ struct AddSmem {
     int32_t bcol[ADD_T + 2];
     int32_t arp[ADD_T + 4];
     int32_t brp[ADD_T + 4];
-    V aval[FILL ? ADD_T + 2 : 1];
-    V bval[FILL ? ADD_T + 2 : 1];
-    int32_t ocol[FILL ? ADD_T + 2 : 1];
-    V oval[FILL ? ADD_T + 2 : 1];
     Split st[ADD_NT + 1];
     int32_t wsum[ADD_NT / 32];
 };
@@ -134,18 +130,18 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
     const int ga0 = s0.a, gb0 = s0.b;
     const int nA = s1.a - ga0, nB = s1.b - gb0;
     const int nrw = min(r1, m - 1) - r0 + 2;  // row offsets r0 .. min(r1, m-1)+1
-    // ---- stage the tile (coalesced) ----
-    for (int i = tid; i < nA; i += ADD_NT) {
-        S.acol[i] = Acol[ga0 + i];
-        if (FILL) S.aval[i] = Aval[ga0 + i];
-    }
-    for (int i = tid; i < nB; i += ADD_NT) {
-        S.bcol[i] = Bcol[gb0 + i];
-        if (FILL) S.bval[i] = Bval[gb0 + i];
-    }
+    // ---- stage the tile (coalesced asynchronous copies, all in flight) ----
+    for (int i = tid; i < nA; i += ADD_NT) cp_async<4>(&S.acol[i], Acol + ga0 + i);
+    for (int i = tid; i < nB; i += ADD_NT) cp_async<4>(&S.bcol[i], Bcol + gb0 + i);
     for (int i = tid; i < nrw; i += ADD_NT) {
-        S.arp[i] = Arp[r0 + i] - ga0;  // tile-relative row offsets
-        S.brp[i] = Brp[r0 + i] - gb0;
+        cp_async<4>(&S.arp[i], Arp + r0 + i);
+        cp_async<4>(&S.brp[i], Brp + r0 + i);
+    }
+    cp_async_wait_all();
+    __syncthreads();
+    for (int i = tid; i < nrw; i += ADD_NT) {  // tile-relative row offsets
+        S.arp[i] -= ga0;
+        S.brp[i] -= gb0;
     }
     __syncthreads();
     const int nrows = r1 - r0;  // row-end items in the tile
@@ -243,23 +239,21 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
         walk([&](int, int, int) { ++cnt; }, [&](int) {});
         int tot;
         const int off = block_exclusive_sum<int, ADD_NT / 32>(cnt, S.wsum, 0, &tot);
-        int o = off;
+        // outputs of this thread are consecutive in C: store them directly
+        // (values read from global at the matched positions, L1-resident)
+        const int64_t base = tile_off[k] + off;
+        int o = 0;
         walk(
             [&](int c, int ia, int ib) {
-                S.ocol[o] = c;
                 V v;
-                if (ia >= 0 && ib >= 0) v = S.aval[ia] + S.bval[ib];  // one rounding, A first
-                else v = (ia >= 0) ? S.aval[ia] : S.bval[ib];
-                S.oval[o] = v;
+                if (ia >= 0 && ib >= 0) v = Aval[ga0 + ia] + Bval[gb0 + ib];  // one rounding, A first
+                else v = (ia >= 0) ? Aval[ga0 + ia] : Bval[gb0 + ib];
+                Ccol[base + o] = c;
+                Cval[base + o] = v;
                 ++o;
             },
             [&](int) {});
-        __syncthreads();
-        const int64_t base = tile_off[k];
-        for (int i = tid; i < tot; i += ADD_NT) {
-            Ccol[base + i] = S.ocol[i];
-            Cval[base + i] = S.oval[i];
-        }
+        (void)tot;
     }
 }
 

@@ -449,16 +449,20 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                     if ((mask >> k) & 1u) run = 0.0;
                 }
                 if (mask) {
-                    // row partials back into this lane's own product slots
+                    // pick row partials from registers (no shared-memory round
+                    // trip: the L1/shared data pipe is the kernel's limit)
+                    auto pick = [&](int kk) {
+                        double r = ev[0];
 #pragma unroll
-                    for (int i = 0; i < K / 2; ++i)
-                        reinterpret_cast<double2 *>(myp)[i ^ s_sw] = make_double2(ev[2 * i], ev[2 * i + 1]);
+                        for (int k = 1; k < K; ++k) r = (k == kk) ? ev[k] : r;
+                        return r;
+                    };
                     const int k0 = __ffs(mask) - 1;
-                    first_v = myp[(((k0 >> 1) ^ s_sw) << 1) | (k0 & 1)];
+                    first_v = pick(k0);
                     first_r = tile_is + int(rmap[qs + k0]) - 1;
                     for (unsigned rest = mask & (mask - 1); rest; rest &= rest - 1) {
                         const int k = __ffs(rest) - 1;
-                        y[tile_is + int(rmap[qs + k]) - 1] = V(myp[(((k >> 1) ^ s_sw) << 1) | (k & 1)]);
+                        y[tile_is + int(rmap[qs + k]) - 1] = V(pick(k));
                     }
                 }
             }
