@@ -19,21 +19,21 @@ namespace msp {
 // stride of the blocked layout).
 __device__ __forceinline__ int sort_pad(int i) { return i + (i >> 4); }
 
-template <int NT, int IPT>
+template <int NT, int IPT, typename KT = uint64_t>
 struct BlockSortSmem {
-    uint64_t keys[NT * IPT + (NT * IPT) / 16 + 2];
+    KT keys[NT * IPT + (NT * IPT) / 16 + 2];
     int vals[NT * IPT + (NT * IPT) / 16 + 2];
 };
 
-template <int IPT>
-__device__ __forceinline__ void thread_sort(uint64_t (&k)[IPT], int (&v)[IPT])
+template <int IPT, typename KT>
+__device__ __forceinline__ void thread_sort(KT (&k)[IPT], int (&v)[IPT])
 {
 #pragma unroll
     for (int r = 0; r < IPT; ++r) {
 #pragma unroll
         for (int i = (r & 1); i + 1 < IPT; i += 2) {
             if (k[i] > k[i + 1]) {
-                const uint64_t tk = k[i];
+                const KT tk = k[i];
                 k[i] = k[i + 1];
                 k[i + 1] = tk;
                 const int tv = v[i];
@@ -47,11 +47,12 @@ __device__ __forceinline__ void thread_sort(uint64_t (&k)[IPT], int (&v)[IPT])
 // Sorts NT*IPT (key, val) items held IPT per thread (any assignment of items
 // to threads); on return thread t holds sorted items [t*IPT, (t+1)*IPT).
 // All NT threads of the CTA must call (uses __syncthreads).
-template <int NT, int IPT>
-__device__ __forceinline__ void block_merge_sort(uint64_t (&k)[IPT], int (&v)[IPT], BlockSortSmem<NT, IPT> &S)
+template <int NT, int IPT, typename KT>
+__device__ __forceinline__ void block_merge_sort(KT (&k)[IPT], int (&v)[IPT], BlockSortSmem<NT, IPT, KT> &S)
 {
     const int tid = threadIdx.x;
-    thread_sort<IPT>(k, v);
+    constexpr KT KMAX = ~KT(0);
+    thread_sort<IPT, KT>(k, v);
 #pragma unroll 1
     for (int w = 1; w < NT; w <<= 1) {
 #pragma unroll
@@ -71,8 +72,8 @@ __device__ __forceinline__ void block_merge_sort(uint64_t (&k)[IPT], int (&v)[IP
             else hi = mid;
         }
         int ia = lo, ib = d - lo;
-        uint64_t ka = ia < la ? S.keys[sort_pad(g0 + ia)] : ~0ull;
-        uint64_t kb = ib < lb ? S.keys[sort_pad(g0 + la + ib)] : ~0ull;
+        KT ka = ia < la ? S.keys[sort_pad(g0 + ia)] : KMAX;
+        KT kb = ib < lb ? S.keys[sort_pad(g0 + la + ib)] : KMAX;
 #pragma unroll
         for (int i = 0; i < IPT; ++i) {
             const bool takea = (ib >= lb) || (ia < la && ka <= kb);
@@ -80,12 +81,12 @@ __device__ __forceinline__ void block_merge_sort(uint64_t (&k)[IPT], int (&v)[IP
                 k[i] = ka;
                 v[i] = S.vals[sort_pad(g0 + ia)];
                 ++ia;
-                ka = ia < la ? S.keys[sort_pad(g0 + ia)] : ~0ull;
+                ka = ia < la ? S.keys[sort_pad(g0 + ia)] : KMAX;
             } else {
                 k[i] = kb;
                 v[i] = S.vals[sort_pad(g0 + la + ib)];
                 ++ib;
-                kb = ib < lb ? S.keys[sort_pad(g0 + la + ib)] : ~0ull;
+                kb = ib < lb ? S.keys[sort_pad(g0 + la + ib)] : KMAX;
             }
         }
         __syncthreads();

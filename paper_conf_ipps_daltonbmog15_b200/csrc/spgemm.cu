@@ -186,7 +186,10 @@ __global__ void gemm_partition_kernel(int32_t m, int64_t nnzA, int64_t nprods, c
 
 template <typename V, bool NUM>
 struct TileSmem {
-    BlockSortSmem<GM_NT, GM_IPT> sort;  // sort.keys doubles as the expansion staging buffer
+    union {
+        BlockSortSmem<GM_NT, GM_IPT, uint64_t> s64;  // s64.keys doubles as the expansion staging buffer
+        BlockSortSmem<GM_NT, GM_IPT, uint32_t> s32;
+    } sort;
     double vals[NUM ? GM_T : 1];
     uint64_t edge_first[GM_NT];
     uint64_t edge_last[GM_NT];
@@ -194,13 +197,147 @@ struct TileSmem {
     int32_t wsum[GM_NT / 32];
 };
 
-// One CTA per tile: expand -> sort by (row, col) -> compress.
+// Key layouts: 64-bit (row offset << 32 | col) always works; 32-bit
+// (row offset << cbits | col) is used when the tile's row span fits, halving
+// the sort's shared-memory traffic and compare cost.
+template <typename KT>
+struct KeyOps;
+template <>
+struct KeyOps<uint64_t> {
+    static constexpr uint64_t MASKED = ~0ull;
+    static constexpr uint64_t NONE = 1ull << 63;  // never equal to a real key
+    __device__ static uint32_t row(uint64_t k, int) { return uint32_t(k >> 32); }
+    __device__ static uint32_t col(uint64_t k, int) { return uint32_t(k); }
+};
+template <>
+struct KeyOps<uint32_t> {
+    static constexpr uint32_t MASKED = ~0u;
+    static constexpr uint32_t NONE = ~0u - 1u;  // real keys stay below (see use32)
+    __device__ static uint32_t row(uint32_t k, int cb) { return k >> cb; }
+    __device__ static uint32_t col(uint32_t k, int cb) { return k & ((1u << cb) - 1u); }
+};
+
+// Sort the staged products by key (stable) and compress (see kernel).
+template <typename KT, typename V, bool NUM>
+__device__ __forceinline__ void sort_compress(TileSmem<V, NUM> &Sm, int np, int32_t rbase, int cbits,
+                                              int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol,
+                                              V *__restrict__ Cval)
+{
+    using O = KeyOps<KT>;
+    const int tid = threadIdx.x;
+    KT k[GM_IPT];
+    int v[GM_IPT];
+#pragma unroll
+    for (int u = 0; u < GM_IPT; ++u) {
+        const int slot = tid + u * GM_NT;
+        const uint64_t k64 = slot < np ? Sm.sort.s64.keys[slot] : KEY_MASKED;
+        if (sizeof(KT) == 8) {
+            k[u] = KT(k64);
+        } else {
+            k[u] = (k64 == KEY_MASKED) ? KT(O::MASKED) : KT((uint32_t(k64 >> 32) << cbits) | uint32_t(k64));
+        }
+        v[u] = slot;
+    }
+    __syncthreads();  // staging is reused by the sort
+    BlockSortSmem<GM_NT, GM_IPT, KT> *ss;
+    if constexpr (sizeof(KT) == 8) ss = &Sm.sort.s64;
+    else ss = &Sm.sort.s32;
+    block_merge_sort<GM_NT, GM_IPT, KT>(k, v, *ss);
+    // neighbours across thread boundaries
+    Sm.edge_first[tid] = k[0];
+    Sm.edge_last[tid] = k[GM_IPT - 1];
+    __syncthreads();
+    const KT prevk = tid > 0 ? KT(Sm.edge_last[tid - 1]) : O::NONE;
+    const KT nextk = tid + 1 < GM_NT ? KT(Sm.edge_first[tid + 1]) : O::NONE;
+    auto newrow = [&](KT pk, KT kk) { return pk == O::MASKED || pk == O::NONE || O::row(pk, cbits) != O::row(kk, cbits); };
+
+    if (!NUM) {
+        // ---- unique count per row (rows are complete in the tile) ----
+        KT pk = prevk;
+        int cnt = 0;
+        int64_t row = -1;
+#pragma unroll
+        for (int i = 0; i < GM_IPT; ++i) {
+            if (k[i] != O::MASKED) {
+                const int64_t r = int64_t(rbase) + int64_t(O::row(k[i], cbits));
+                if (r != row) {
+                    if (cnt) atomicAdd(&Crp[row + 1], cnt);
+                    cnt = 0;
+                    row = r;
+                }
+                if (k[i] != pk) ++cnt;
+            }
+            pk = k[i];
+        }
+        if (cnt) atomicAdd(&Crp[row + 1], cnt);
+    } else {
+        // ---- unique (col, sum): position = C.rp[row] + rank of the key in its row ----
+        int heads = 0, last_rs = -1;  // heads in this thread; heads before its last row start
+        double trail = 0.0;           // sum after the last head in this thread
+        {
+            KT pk = prevk;
+#pragma unroll
+            for (int i = 0; i < GM_IPT; ++i) {
+                if (k[i] != O::MASKED) {
+                    const double val = Sm.vals[v[i]];
+                    if (k[i] != pk) {
+                        if (newrow(pk, k[i])) last_rs = heads;
+                        ++heads;
+                        trail = val;
+                    } else {
+                        trail = trail + val;
+                    }
+                }
+                pk = k[i];
+            }
+        }
+        int tot;
+        const int u0 = block_exclusive_sum<int, GM_NT / 32>(heads, Sm.wsum, 0, &tot);
+        SegPair<double> all;
+        const SegPair<double> carry =
+            block_seg_exclusive<double, GM_NT / 32>(SegPair<double>{heads > 0, trail}, SegPair<double>{0, 0.0},
+                                                    Sm.scan_w, 0, &all);
+        // tile rank of the first key of the row open at this thread's start
+        const int rs_carry = block_exclusive_max<GM_NT / 32>(last_rs >= 0 ? u0 + last_rs : -1, Sm.wsum, 0);
+        KT pk = prevk;
+        int u = u0 - 1, row_u = rs_carry;
+        double run = carry.v;
+#pragma unroll
+        for (int i = 0; i < GM_IPT; ++i) {
+            if (k[i] != O::MASKED) {
+                const double val = Sm.vals[v[i]];
+                if (k[i] != pk) {
+                    ++u;
+                    if (newrow(pk, k[i])) row_u = u;
+                    run = val;
+                } else {
+                    run = run + val;
+                }
+                const KT nk = (i + 1 < GM_IPT) ? k[i + 1] : nextk;
+                if (nk != k[i]) {  // run ends here
+                    const int64_t row = int64_t(rbase) + int64_t(O::row(k[i], cbits));
+                    const int64_t pos = int64_t(Crp[row]) + (u - row_u);
+                    Ccol[pos] = int32_t(O::col(k[i], cbits));
+                    Cval[pos] = V(run);
+                }
+            }
+            pk = k[i];
+        }
+    }
+}
+
+// One CTA per tile: expand -> sort by (row, col) -> compress.  Products are
+// expanded in merge-path order (each thread finds its split of the tile's
+// (nonzero ends, products) once, then walks), staged by product index, sorted
+// stably (so equal keys stay in k order), reduced with head flags.  Symbolic:
+// unique counts per row into C.row_offsets.  Numeric: (col, sum) at
+// C.row_offsets[row] + rank in row.
 template <typename V, bool NUM>
 __global__ void __launch_bounds__(GM_NT)
 gemm_tile_kernel(const int32_t *__restrict__ Acol, const V *__restrict__ Aval, const int32_t *__restrict__ Brp,
                  const int32_t *__restrict__ Bcol, const V *__restrict__ Bval, const int32_t *__restrict__ arow,
                  const int64_t *__restrict__ S, const uint8_t *__restrict__ rowlong, const GSplit *__restrict__ splits,
-                 int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol, V *__restrict__ Cval)
+                 int cbits, int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol, V *__restrict__ Cval)
 {
     extern __shared__ __align__(16) char smem_raw[];
     TileSmem<V, NUM> &Sm = *reinterpret_cast<TileSmem<V, NUM> *>(smem_raw);
@@ -210,6 +347,7 @@ gemm_tile_kernel(const int32_t *__restrict__ Acol, const V *__restrict__ Aval, c
     const int nz = int(s1.j - j0), np = int(s1.p - p0);
     if (np == 0) return;
     const int32_t rbase = arow[j0];
+    const int32_t rspan = arow[j0 + nz - 1] - rbase + 1;
     // ---- expansion: merge path over (nonzero ends, products) of the tile ----
     {
         const int items = nz + np;
@@ -248,103 +386,15 @@ gemm_tile_kernel(const int32_t *__restrict__ Acol, const V *__restrict__ Aval, c
             }
             const int slot = int(p - p0);
             const int64_t bi = bofs + p;
-            Sm.sort.keys[slot] = masked ? KEY_MASKED : (rowkey | uint32_t(Bcol[bi]));
+            Sm.sort.s64.keys[slot] = masked ? KEY_MASKED : (rowkey | uint32_t(Bcol[bi]));
             if (NUM) Sm.vals[slot] = av * double(Bval[bi]);
             ++p;
         }
     }
     __syncthreads();
-    // ---- sort the tile's products by (row, col), stable ----
-    uint64_t k[GM_IPT];
-    int v[GM_IPT];
-#pragma unroll
-    for (int u = 0; u < GM_IPT; ++u) {
-        const int slot = tid + u * GM_NT;
-        k[u] = slot < np ? Sm.sort.keys[slot] : KEY_MASKED;
-        v[u] = slot;
-    }
-    __syncthreads();  // staging is reused by the sort
-    block_merge_sort<GM_NT, GM_IPT>(k, v, Sm.sort);
-    // neighbours across thread boundaries
-    Sm.edge_first[tid] = k[0];
-    Sm.edge_last[tid] = k[GM_IPT - 1];
-    __syncthreads();
-    const uint64_t prevk = tid > 0 ? Sm.edge_last[tid - 1] : KEY_NONE;
-    const uint64_t nextk = tid + 1 < GM_NT ? Sm.edge_first[tid + 1] : KEY_NONE;
-
-    if (!NUM) {
-        // ---- unique count per row (rows are complete in the tile) ----
-        uint64_t pk = prevk;
-        int cnt = 0;
-        int64_t row = -1;
-#pragma unroll
-        for (int i = 0; i < GM_IPT; ++i) {
-            if (k[i] != KEY_MASKED) {
-                const int64_t r = int64_t(rbase) + int64_t(k[i] >> 32);
-                if (r != row) {
-                    if (cnt) atomicAdd(&Crp[row + 1], cnt);
-                    cnt = 0;
-                    row = r;
-                }
-                if (k[i] != pk) ++cnt;
-            }
-            pk = k[i];
-        }
-        if (cnt) atomicAdd(&Crp[row + 1], cnt);
-    } else {
-        // ---- unique (col, sum): position = C.rp[row] + rank of the key in its row ----
-        int heads = 0, last_rs = -1;  // heads in this thread; heads before its last row start
-        double trail = 0.0;           // sum after the last head in this thread
-        {
-            uint64_t pk = prevk;
-#pragma unroll
-            for (int i = 0; i < GM_IPT; ++i) {
-                if (k[i] != KEY_MASKED) {
-                    const double val = Sm.vals[v[i]];
-                    if (k[i] != pk) {
-                        if (pk == KEY_MASKED || pk == KEY_NONE || (pk >> 32) != (k[i] >> 32)) last_rs = heads;
-                        ++heads;
-                        trail = val;
-                    } else {
-                        trail = trail + val;
-                    }
-                }
-                pk = k[i];
-            }
-        }
-        int tot;
-        const int u0 = block_exclusive_sum<int, GM_NT / 32>(heads, Sm.wsum, 0, &tot);
-        SegPair<double> all;
-        const SegPair<double> carry =
-            block_seg_exclusive<double, GM_NT / 32>(SegPair<double>{heads > 0, trail}, SegPair<double>{0, 0.0},
-                                                    Sm.scan_w, 0, &all);
-        // tile rank of the first key of the row open at this thread's start
-        const int rs_carry = block_exclusive_max<GM_NT / 32>(last_rs >= 0 ? u0 + last_rs : -1, Sm.wsum, 0);
-        uint64_t pk = prevk;
-        int u = u0 - 1, row_u = rs_carry;
-        double run = carry.v;
-#pragma unroll
-        for (int i = 0; i < GM_IPT; ++i) {
-            if (k[i] != KEY_MASKED) {
-                const double val = Sm.vals[v[i]];
-                if (k[i] != pk) {
-                    ++u;
-                    if (pk == KEY_MASKED || pk == KEY_NONE || (pk >> 32) != (k[i] >> 32)) row_u = u;
-                    run = val;
-                } else {
-                    run = run + val;
-                }
-                const uint64_t nk = (i + 1 < GM_IPT) ? k[i + 1] : nextk;
-                if (nk != k[i]) {  // run ends here
-                    const int64_t row = int64_t(rbase) + int64_t(k[i] >> 32);
-                    const int64_t pos = int64_t(Crp[row]) + (u - row_u);
-                    Ccol[pos] = int32_t(uint32_t(k[i]));
-                    Cval[pos] = V(run);
-                }
-            }
-            pk = k[i];
-        }
-    }
+    const bool use32 = cbits < 31 && (int64_t(rspan) + 2 <= (int64_t(1) << (32 - cbits)));
+    if (use32) sort_compress<uint32_t, V, NUM>(Sm, np, rbase, cbits, Crp, Ccol, Cval);
+    else sort_compress<uint64_t, V, NUM>(Sm, np, rbase, cbits, Crp, Ccol, Cval);
 }
 
 // ---------------------------------------------------------- long rows ----
@@ -611,9 +661,11 @@ msp_status run_tiles(const msp_csr *A, const msp_csr *B, const SetupWs &sw, cons
         configured = 1;
     }
     if (ntiles <= 0) return MSP_OK;
+    int cbits = 1;
+    while (cbits < 31 && (int64_t(1) << cbits) < int64_t(B->ncols)) ++cbits;
     kern<<<unsigned(ntiles), GM_NT, smem, s>>>(A->col_idx, static_cast<const V *>(A->vals), B->row_offsets,
                                                 B->col_idx, static_cast<const V *>(B->vals), sw.arow, sw.S,
-                                                sw.rowlong, mw.splits, Crp, Ccol, static_cast<V *>(Cval));
+                                                sw.rowlong, mw.splits, cbits, Crp, Ccol, static_cast<V *>(Cval));
     return last_launch("gemm_tile_kernel");
 }
 
