@@ -74,20 +74,19 @@ __device__ __forceinline__ void block_merge_sort(KT (&k)[IPT], int (&v)[IPT], Bl
         int ia = lo, ib = d - lo;
         KT ka = ia < la ? S.keys[sort_pad(g0 + ia)] : KMAX;
         KT kb = ib < lb ? S.keys[sort_pad(g0 + la + ib)] : KMAX;
+        // branch-free serial merge (lanes of a warp take different sides)
 #pragma unroll
         for (int i = 0; i < IPT; ++i) {
             const bool takea = (ib >= lb) || (ia < la && ka <= kb);
-            if (takea) {
-                k[i] = ka;
-                v[i] = S.vals[sort_pad(g0 + ia)];
-                ++ia;
-                ka = ia < la ? S.keys[sort_pad(g0 + ia)] : KMAX;
-            } else {
-                k[i] = kb;
-                v[i] = S.vals[sort_pad(g0 + la + ib)];
-                ++ib;
-                kb = ib < lb ? S.keys[sort_pad(g0 + la + ib)] : KMAX;
-            }
+            const int src = takea ? (g0 + ia) : (g0 + la + ib);
+            k[i] = takea ? ka : kb;
+            v[i] = S.vals[sort_pad(src)];
+            ia += takea ? 1 : 0;
+            ib += takea ? 0 : 1;
+            const bool more = takea ? (ia < la) : (ib < lb);
+            const KT kn = more ? S.keys[sort_pad(src + 1)] : KMAX;
+            ka = takea ? kn : ka;
+            kb = takea ? kb : kn;
         }
         __syncthreads();
     }
