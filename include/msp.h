@@ -153,8 +153,14 @@ msp_status msp_spadd_numeric(const msp_csr *A, const msp_csr *B, const int32_t *
  * tile boundary and rows longer than a tile are completed by a second pass
  * (the paper's global phase).  Writes C_row_offsets and
  * *nnzC_host; synchronises.  MSP_ERR_OVERFLOW if nnz(C) > INT32_MAX.
- * Numeric: same passes with values; writes C_col_idx / C_vals; fp64
- * accumulation in product order (k ascending).  Async.
+ * The symbolic pass keeps every tile's sorting permutation in main_ws
+ * (2 bytes per tile slot, as the paper stores the CTA sort's permutation,
+ * P:1140-1175).
+ * Numeric: re-expands the products with values, applies the stored
+ * permutation (no second sort) and compresses; the long-row pass is repeated
+ * with values.  Writes C_col_idx / C_vals; fp64 accumulation in a fixed,
+ * deterministic order.  Must follow msp_spgemm_symbolic on the same main_ws
+ * with A and B unchanged.  Async.
  * setup_ws: msp_spgemm_setup_workspace() bytes; main_ws: info.main_ws_bytes.
  * ------------------------------------------------------------------------ */
 typedef struct {

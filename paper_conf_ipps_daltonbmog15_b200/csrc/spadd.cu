@@ -257,11 +257,6 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
     }
 }
 
-__global__ void check_total_kernel(const int64_t *tile_total, const int64_t *row_total, int32_t *ok)
-{
-    *ok = (*tile_total == *row_total) ? 1 : 0;
-}
-
 struct AddWs {
     Split *splits;
     int32_t *tile_count;

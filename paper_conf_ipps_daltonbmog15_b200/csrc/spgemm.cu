@@ -48,7 +48,6 @@ constexpr int GM_LONG = GM_T / 4;     // rows with more items than this are long
 constexpr int GM_TP = GM_T - GM_LONG;
 constexpr int GM_TL = GM_T;           // products per long-row chunk
 constexpr uint64_t KEY_MASKED = ~0ull;
-constexpr uint64_t KEY_NONE = 1ull << 63;  // never equal to a real key
 
 __device__ __forceinline__ int64_t dmin(int64_t a, int64_t b) { return a < b ? a : b; }
 __device__ __forceinline__ int64_t dmax(int64_t a, int64_t b) { return a > b ? a : b; }
@@ -217,32 +216,54 @@ struct KeyOps<uint32_t> {
     __device__ static uint32_t col(uint32_t k, int cb) { return k & ((1u << cb) - 1u); }
 };
 
-// Sort the staged products by key (stable) and compress (see kernel).
+// Symbolic: sort the staged products by key and store the tile's sorting
+// permutation; numeric: apply the stored permutation instead of sorting
+// again (the paper keeps the CTA sort's permutation in global memory and
+// re-expands the products into it).  Then compress (see kernel).
 template <typename KT, typename V, bool NUM>
 __device__ __forceinline__ void sort_compress(TileSmem<V, NUM> &Sm, int np, int32_t rbase, int cbits,
-                                              int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol,
-                                              V *__restrict__ Cval)
+                                              uint16_t *__restrict__ tperm, int32_t *__restrict__ Crp,
+                                              int32_t *__restrict__ Ccol, V *__restrict__ Cval)
 {
     using O = KeyOps<KT>;
     const int tid = threadIdx.x;
     KT k[GM_IPT];
     int v[GM_IPT];
-#pragma unroll
-    for (int u = 0; u < GM_IPT; ++u) {
-        const int slot = tid + u * GM_NT;
+    auto key_of = [&](int slot) -> KT {
         const uint64_t k64 = slot < np ? Sm.sort.s64.keys[slot] : KEY_MASKED;
-        if (sizeof(KT) == 8) {
-            k[u] = KT(k64);
-        } else {
-            k[u] = (k64 == KEY_MASKED) ? KT(O::MASKED) : KT((uint32_t(k64 >> 32) << cbits) | uint32_t(k64));
+        if constexpr (sizeof(KT) == 8) return KT(k64);
+        else return (k64 == KEY_MASKED) ? KT(O::MASKED) : KT((uint32_t(k64 >> 32) << cbits) | uint32_t(k64));
+    };
+    static_assert(GM_IPT == 16 && GM_T <= 65536, "permutation packing");
+    uint4 *pp = reinterpret_cast<uint4 *>(tperm + tid * GM_IPT);
+    if constexpr (!NUM) {
+#pragma unroll
+        for (int u = 0; u < GM_IPT; ++u) {
+            const int slot = tid + u * GM_NT;
+            k[u] = key_of(slot);
+            v[u] = slot;
         }
-        v[u] = slot;
+        __syncthreads();  // staging is reused by the sort
+        BlockSortSmem<GM_NT, GM_IPT, KT> *ss;
+        if constexpr (sizeof(KT) == 8) ss = &Sm.sort.s64;
+        else ss = &Sm.sort.s32;
+        block_merge_sort<GM_NT, GM_IPT, KT>(k, v, *ss);
+        uint32_t w[GM_IPT / 2];
+#pragma unroll
+        for (int i = 0; i < GM_IPT / 2; ++i) w[i] = uint32_t(v[2 * i]) | (uint32_t(v[2 * i + 1]) << 16);
+        pp[0] = make_uint4(w[0], w[1], w[2], w[3]);
+        pp[1] = make_uint4(w[4], w[5], w[6], w[7]);
+    } else {
+        const uint4 q0 = pp[0], q1 = pp[1];
+        const uint32_t w[GM_IPT / 2] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w};
+#pragma unroll
+        for (int i = 0; i < GM_IPT; ++i) {
+            const int pos = tid * GM_IPT + i;
+            const int slot = int((w[i >> 1] >> ((i & 1) * 16)) & 0xffffu);
+            k[i] = pos < np ? key_of(slot) : KT(O::MASKED);
+            v[i] = slot;
+        }
     }
-    __syncthreads();  // staging is reused by the sort
-    BlockSortSmem<GM_NT, GM_IPT, KT> *ss;
-    if constexpr (sizeof(KT) == 8) ss = &Sm.sort.s64;
-    else ss = &Sm.sort.s32;
-    block_merge_sort<GM_NT, GM_IPT, KT>(k, v, *ss);
     // neighbours across thread boundaries
     Sm.edge_first[tid] = k[0];
     Sm.edge_last[tid] = k[GM_IPT - 1];
@@ -337,7 +358,8 @@ __global__ void __launch_bounds__(GM_NT)
 gemm_tile_kernel(const int32_t *__restrict__ Acol, const V *__restrict__ Aval, const int32_t *__restrict__ Brp,
                  const int32_t *__restrict__ Bcol, const V *__restrict__ Bval, const int32_t *__restrict__ arow,
                  const int64_t *__restrict__ S, const uint8_t *__restrict__ rowlong, const GSplit *__restrict__ splits,
-                 int cbits, int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol, V *__restrict__ Cval)
+                 int cbits, uint16_t *__restrict__ perm, int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol,
+                 V *__restrict__ Cval)
 {
     extern __shared__ __align__(16) char smem_raw[];
     TileSmem<V, NUM> &Sm = *reinterpret_cast<TileSmem<V, NUM> *>(smem_raw);
@@ -393,8 +415,9 @@ gemm_tile_kernel(const int32_t *__restrict__ Acol, const V *__restrict__ Aval, c
     }
     __syncthreads();
     const bool use32 = cbits < 31 && (int64_t(rspan) + 2 <= (int64_t(1) << (32 - cbits)));
-    if (use32) sort_compress<uint32_t, V, NUM>(Sm, np, rbase, cbits, Crp, Ccol, Cval);
-    else sort_compress<uint64_t, V, NUM>(Sm, np, rbase, cbits, Crp, Ccol, Cval);
+    uint16_t *tperm = perm + size_t(blockIdx.x) * GM_T;
+    if (use32) sort_compress<uint32_t, V, NUM>(Sm, np, rbase, cbits, tperm, Crp, Ccol, Cval);
+    else sort_compress<uint64_t, V, NUM>(Sm, np, rbase, cbits, tperm, Crp, Ccol, Cval);
 }
 
 // ---------------------------------------------------------- long rows ----
@@ -592,6 +615,7 @@ __global__ void long_emit_kernel(int64_t LP, int64_t nlong, const int64_t *__res
 
 struct MainWs {
     GSplit *splits;
+    uint16_t *perm;  // per tile: the symbolic sort's permutation (GM_T entries)
     int32_t *Xc[2];
     double *Xv[2];
     int32_t *heads;
@@ -607,6 +631,7 @@ MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, void *ws, size_t cap, b
     MainWs w;
     Carve cv(ws, cap);
     w.splits = cv.take<GSplit>(size_t(ntiles + 1));
+    w.perm = cv.take<uint16_t>(size_t(ntiles) * GM_T);
     for (int i = 0; i < 2; ++i) {
         w.Xc[i] = cv.take<int32_t>(size_t(LP > 0 ? LP : 1));
         w.Xv[i] = cv.take<double>(size_t(LP > 0 ? LP : 1));
@@ -665,7 +690,7 @@ msp_status run_tiles(const msp_csr *A, const msp_csr *B, const SetupWs &sw, cons
     while (cbits < 31 && (int64_t(1) << cbits) < int64_t(B->ncols)) ++cbits;
     kern<<<unsigned(ntiles), GM_NT, smem, s>>>(A->col_idx, static_cast<const V *>(A->vals), B->row_offsets,
                                                 B->col_idx, static_cast<const V *>(B->vals), sw.arow, sw.S,
-                                                sw.rowlong, mw.splits, cbits, Crp, Ccol, static_cast<V *>(Cval));
+                                                sw.rowlong, mw.splits, cbits, mw.perm, Crp, Ccol, static_cast<V *>(Cval));
     return last_launch("gemm_tile_kernel");
 }
 
