@@ -183,45 +183,84 @@ __global__ void gemm_partition_kernel(int32_t m, int64_t nnzA, int64_t nprods, c
     }
 }
 
-template <typename V, bool NUM>
-struct TileSmem {
-    union {
-        BlockSortSmem<GM_NT, GM_IPT, uint64_t> s64;  // s64.keys doubles as the expansion staging buffer
-        BlockSortSmem<GM_NT, GM_IPT, uint32_t> s32;
-    } sort;
-    double vals[NUM ? GM_T : 1];
-    uint64_t edge_first[GM_NT];
-    uint64_t edge_last[GM_NT];
-    SegPair<double> scan_w[GM_NT / 32];
-    int32_t wsum[GM_NT / 32];
-};
-
 // Key layouts: 64-bit (row offset << 32 | col) always works; 32-bit
-// (row offset << cbits | col) is used when the tile's row span fits, halving
-// the sort's shared-memory traffic and compare cost.
+// (row offset << cbits | col) is used when every tile's row span fits,
+// halving the staging / sort shared memory (2 CTAs per SM) and compare cost.
 template <typename KT>
 struct KeyOps;
 template <>
 struct KeyOps<uint64_t> {
     static constexpr uint64_t MASKED = ~0ull;
     static constexpr uint64_t NONE = 1ull << 63;  // never equal to a real key
+    __device__ static uint64_t make(uint32_t r, uint32_t c, int) { return (uint64_t(r) << 32) | c; }
     __device__ static uint32_t row(uint64_t k, int) { return uint32_t(k >> 32); }
     __device__ static uint32_t col(uint64_t k, int) { return uint32_t(k); }
 };
 template <>
 struct KeyOps<uint32_t> {
     static constexpr uint32_t MASKED = ~0u;
-    static constexpr uint32_t NONE = ~0u - 1u;  // real keys stay below (see use32)
+    static constexpr uint32_t NONE = ~0u - 1u;  // real keys stay below (tile_span_ok)
+    __device__ static uint32_t make(uint32_t r, uint32_t c, int cb) { return (r << cb) | c; }
     __device__ static uint32_t row(uint32_t k, int cb) { return k >> cb; }
     __device__ static uint32_t col(uint32_t k, int cb) { return k & ((1u << cb) - 1u); }
 };
 
-// Symbolic: sort the staged products by key and store the tile's sorting
-// permutation; numeric: apply the stored permutation instead of sorting
-// again (the paper keeps the CTA sort's permutation in global memory and
-// re-expands the products into it).  Then compress (see kernel).
-template <typename KT, typename V, bool NUM>
-__device__ __forceinline__ void sort_compress(TileSmem<V, NUM> &Sm, int np, int32_t rbase, int cbits,
+// Shared memory of one tile.  Symbolic: the staging buffer (keys by product
+// slot) is reused by the sort.  Numeric: staging keys + product values only
+// (the permutation comes from the symbolic pass).
+template <typename KT, bool NUM>
+struct TileKeys {
+    union {
+        KT stage[GM_T];
+        BlockSortSmem<GM_NT, GM_IPT, KT> sort;
+    };
+};
+template <typename KT>
+struct TileKeys<KT, true> {
+    KT stage[GM_T];
+};
+template <typename KT, bool NUM>
+struct TileSmem {
+    TileKeys<KT, NUM> keys;
+    double vals[NUM ? GM_T : 1];
+    KT edge_first[GM_NT];
+    KT edge_last[GM_NT];
+    SegPair<double> scan_w[GM_NT / 32];
+    int32_t wsum[GM_NT / 32];
+};
+
+__device__ __forceinline__ unsigned long long warp_reduce_max_u64(unsigned long long v)
+{
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const unsigned long long t = __shfl_xor_sync(0xffffffffu, v, o);
+        v = v > t ? v : t;
+    }
+    return v;
+}
+
+// Largest row span of any tile (decides the key width for the whole launch).
+__global__ void tile_span_kernel(int64_t ntiles, const GSplit *__restrict__ splits, const int32_t *__restrict__ arow,
+                                 unsigned long long *__restrict__ maxspan)
+{
+    unsigned long long mx = 0;
+    for (int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; k < ntiles; k += int64_t(gridDim.x) * blockDim.x) {
+        const GSplit s0 = splits[k], s1 = splits[k + 1];
+        if (s1.p == s0.p) continue;
+        const int64_t nz = s1.j - s0.j;
+        const int64_t span = nz > 0 ? int64_t(arow[s0.j + nz - 1]) - arow[s0.j] + 1 : 1;
+        mx = mx > (unsigned long long)span ? mx : (unsigned long long)span;
+    }
+    mx = warp_reduce_max_u64(mx);
+    if ((threadIdx.x & 31) == 0 && mx) atomicMax(maxspan, mx);
+}
+
+// Symbolic: sort the staged keys and store the tile's sorting permutation;
+// numeric: apply the stored permutation instead of sorting again (the paper
+// keeps the CTA sort's permutation in global memory and re-expands the
+// products into it).  Then compress (see kernel).
+template <typename KT, bool NUM, typename V>
+__device__ __forceinline__ void sort_compress(TileSmem<KT, NUM> &Sm, int np, int32_t rbase, int cbits,
                                               uint16_t *__restrict__ tperm, int32_t *__restrict__ Crp,
                                               int32_t *__restrict__ Ccol, V *__restrict__ Cval)
 {
@@ -229,25 +268,17 @@ __device__ __forceinline__ void sort_compress(TileSmem<V, NUM> &Sm, int np, int3
     const int tid = threadIdx.x;
     KT k[GM_IPT];
     int v[GM_IPT];
-    auto key_of = [&](int slot) -> KT {
-        const uint64_t k64 = slot < np ? Sm.sort.s64.keys[slot] : KEY_MASKED;
-        if constexpr (sizeof(KT) == 8) return KT(k64);
-        else return (k64 == KEY_MASKED) ? KT(O::MASKED) : KT((uint32_t(k64 >> 32) << cbits) | uint32_t(k64));
-    };
     static_assert(GM_IPT == 16 && GM_T <= 65536, "permutation packing");
     uint4 *pp = reinterpret_cast<uint4 *>(tperm + tid * GM_IPT);
     if constexpr (!NUM) {
 #pragma unroll
         for (int u = 0; u < GM_IPT; ++u) {
             const int slot = tid + u * GM_NT;
-            k[u] = key_of(slot);
+            k[u] = slot < np ? Sm.keys.stage[slot] : O::MASKED;
             v[u] = slot;
         }
         __syncthreads();  // staging is reused by the sort
-        BlockSortSmem<GM_NT, GM_IPT, KT> *ss;
-        if constexpr (sizeof(KT) == 8) ss = &Sm.sort.s64;
-        else ss = &Sm.sort.s32;
-        block_merge_sort<GM_NT, GM_IPT, KT>(k, v, *ss);
+        block_merge_sort<GM_NT, GM_IPT, KT>(k, v, Sm.keys.sort);
         uint32_t w[GM_IPT / 2];
 #pragma unroll
         for (int i = 0; i < GM_IPT / 2; ++i) w[i] = uint32_t(v[2 * i]) | (uint32_t(v[2 * i + 1]) << 16);
@@ -260,7 +291,9 @@ __device__ __forceinline__ void sort_compress(TileSmem<V, NUM> &Sm, int np, int3
         for (int i = 0; i < GM_IPT; ++i) {
             const int pos = tid * GM_IPT + i;
             const int slot = int((w[i >> 1] >> ((i & 1) * 16)) & 0xffffu);
-            k[i] = pos < np ? key_of(slot) : KT(O::MASKED);
+            // masked (long-row) products and padding share the MASKED key, so a
+            // position < np may hold a padding slot >= np
+            k[i] = (pos < np && slot < np) ? Sm.keys.stage[slot] : O::MASKED;
             v[i] = slot;
         }
     }
@@ -268,11 +301,11 @@ __device__ __forceinline__ void sort_compress(TileSmem<V, NUM> &Sm, int np, int3
     Sm.edge_first[tid] = k[0];
     Sm.edge_last[tid] = k[GM_IPT - 1];
     __syncthreads();
-    const KT prevk = tid > 0 ? KT(Sm.edge_last[tid - 1]) : O::NONE;
-    const KT nextk = tid + 1 < GM_NT ? KT(Sm.edge_first[tid + 1]) : O::NONE;
+    const KT prevk = tid > 0 ? Sm.edge_last[tid - 1] : O::NONE;
+    const KT nextk = tid + 1 < GM_NT ? Sm.edge_first[tid + 1] : O::NONE;
     auto newrow = [&](KT pk, KT kk) { return pk == O::MASKED || pk == O::NONE || O::row(pk, cbits) != O::row(kk, cbits); };
 
-    if (!NUM) {
+    if constexpr (!NUM) {
         // ---- unique count per row (rows are complete in the tile) ----
         KT pk = prevk;
         int cnt = 0;
@@ -350,26 +383,26 @@ __device__ __forceinline__ void sort_compress(TileSmem<V, NUM> &Sm, int np, int3
 // One CTA per tile: expand -> sort by (row, col) -> compress.  Products are
 // expanded in merge-path order (each thread finds its split of the tile's
 // (nonzero ends, products) once, then walks), staged by product index, sorted
-// stably (so equal keys stay in k order), reduced with head flags.  Symbolic:
-// unique counts per row into C.row_offsets.  Numeric: (col, sum) at
+// (symbolic; the permutation is kept for numeric), reduced with head flags.
+// Symbolic: unique counts per row into C.row_offsets.  Numeric: (col, sum) at
 // C.row_offsets[row] + rank in row.
-template <typename V, bool NUM>
-__global__ void __launch_bounds__(GM_NT)
+template <typename KT, typename V, bool NUM>
+__global__ void __launch_bounds__(GM_NT, 2)
 gemm_tile_kernel(const int32_t *__restrict__ Acol, const V *__restrict__ Aval, const int32_t *__restrict__ Brp,
                  const int32_t *__restrict__ Bcol, const V *__restrict__ Bval, const int32_t *__restrict__ arow,
                  const int64_t *__restrict__ S, const uint8_t *__restrict__ rowlong, const GSplit *__restrict__ splits,
                  int cbits, uint16_t *__restrict__ perm, int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol,
                  V *__restrict__ Cval)
 {
+    using O = KeyOps<KT>;
     extern __shared__ __align__(16) char smem_raw[];
-    TileSmem<V, NUM> &Sm = *reinterpret_cast<TileSmem<V, NUM> *>(smem_raw);
+    TileSmem<KT, NUM> &Sm = *reinterpret_cast<TileSmem<KT, NUM> *>(smem_raw);
     const int tid = threadIdx.x;
     const GSplit s0 = splits[blockIdx.x], s1 = splits[blockIdx.x + 1];
     const int64_t j0 = s0.j, p0 = s0.p;
     const int nz = int(s1.j - j0), np = int(s1.p - p0);
     if (np == 0) return;
     const int32_t rbase = arow[j0];
-    const int32_t rspan = arow[j0 + nz - 1] - rbase + 1;
     // ---- expansion: merge path over (nonzero ends, products) of the tile ----
     {
         const int items = nz + np;
@@ -386,7 +419,7 @@ gemm_tile_kernel(const int32_t *__restrict__ Acol, const V *__restrict__ Aval, c
         const int todo = min(GM_IPT, items - dt);
         int64_t sj1 = (j < jend) ? S[j + 1] : INT64_MAX;
         int64_t bofs = 0;
-        uint64_t rowkey = 0;
+        uint32_t rofs = 0;
         bool masked = true;
         double av = 0.0;
         bool loaded = false;
@@ -400,7 +433,7 @@ gemm_tile_kernel(const int32_t *__restrict__ Acol, const V *__restrict__ Aval, c
             if (!loaded) {
                 const int32_t r = arow[j];
                 masked = rowlong[r] != 0;
-                rowkey = uint64_t(uint32_t(r - rbase)) << 32;
+                rofs = uint32_t(r - rbase);
                 const int32_t kk = Acol[j];
                 bofs = int64_t(Brp[kk]) - S[j];
                 if (NUM) av = double(Aval[j]);
@@ -408,16 +441,13 @@ gemm_tile_kernel(const int32_t *__restrict__ Acol, const V *__restrict__ Aval, c
             }
             const int slot = int(p - p0);
             const int64_t bi = bofs + p;
-            Sm.sort.s64.keys[slot] = masked ? KEY_MASKED : (rowkey | uint32_t(Bcol[bi]));
+            Sm.keys.stage[slot] = masked ? O::MASKED : O::make(rofs, uint32_t(Bcol[bi]), cbits);
             if (NUM) Sm.vals[slot] = av * double(Bval[bi]);
             ++p;
         }
     }
     __syncthreads();
-    const bool use32 = cbits < 31 && (int64_t(rspan) + 2 <= (int64_t(1) << (32 - cbits)));
-    uint16_t *tperm = perm + size_t(blockIdx.x) * GM_T;
-    if (use32) sort_compress<uint32_t, V, NUM>(Sm, np, rbase, cbits, tperm, Crp, Ccol, Cval);
-    else sort_compress<uint64_t, V, NUM>(Sm, np, rbase, cbits, tperm, Crp, Ccol, Cval);
+    sort_compress<KT, NUM, V>(Sm, np, rbase, cbits, perm + size_t(blockIdx.x) * GM_T, Crp, Ccol, Cval);
 }
 
 // ---------------------------------------------------------- long rows ----
@@ -672,12 +702,12 @@ msp_status read_info(const SetupWs &sw, int64_t m, int64_t nnzA, HostInfo *h, cu
     return MSP_OK;
 }
 
-template <typename V, bool NUM>
-msp_status run_tiles(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, int64_t ntiles,
-                     int32_t *Crp, int32_t *Ccol, void *Cval, cudaStream_t s)
+template <typename KT, typename V, bool NUM>
+msp_status launch_tiles(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, int64_t ntiles,
+                        int cbits, int32_t *Crp, int32_t *Ccol, void *Cval, cudaStream_t s)
 {
-    auto kern = gemm_tile_kernel<V, NUM>;
-    const int smem = int(sizeof(TileSmem<V, NUM>));
+    auto kern = gemm_tile_kernel<KT, V, NUM>;
+    const int smem = int(sizeof(TileSmem<KT, NUM>));
     static int configured = 0;
     if (!configured) {
         msp_status st = cuda_check(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem),
@@ -685,13 +715,25 @@ msp_status run_tiles(const msp_csr *A, const msp_csr *B, const SetupWs &sw, cons
         if (st != MSP_OK) return st;
         configured = 1;
     }
+    kern<<<unsigned(ntiles), GM_NT, smem, s>>>(A->col_idx, static_cast<const V *>(A->vals), B->row_offsets,
+                                                B->col_idx, static_cast<const V *>(B->vals), sw.arow, sw.S,
+                                                sw.rowlong, mw.splits, cbits, mw.perm, Crp, Ccol,
+                                                static_cast<V *>(Cval));
+    return last_launch("gemm_tile_kernel");
+}
+
+// Key width for the launch: 32-bit keys when (row offset, col) of every tile
+// fits below the two reserved values, else 64-bit.
+template <typename V, bool NUM>
+msp_status run_tiles(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, int64_t ntiles,
+                     int64_t maxspan, int32_t *Crp, int32_t *Ccol, void *Cval, cudaStream_t s)
+{
     if (ntiles <= 0) return MSP_OK;
     int cbits = 1;
     while (cbits < 31 && (int64_t(1) << cbits) < int64_t(B->ncols)) ++cbits;
-    kern<<<unsigned(ntiles), GM_NT, smem, s>>>(A->col_idx, static_cast<const V *>(A->vals), B->row_offsets,
-                                                B->col_idx, static_cast<const V *>(B->vals), sw.arow, sw.S,
-                                                sw.rowlong, mw.splits, cbits, mw.perm, Crp, Ccol, static_cast<V *>(Cval));
-    return last_launch("gemm_tile_kernel");
+    const bool use32 = cbits < 31 && (maxspan + 2 <= (int64_t(1) << (32 - cbits)));
+    return use32 ? launch_tiles<uint32_t, V, NUM>(A, B, sw, mw, ntiles, cbits, Crp, Ccol, Cval, s)
+                 : launch_tiles<uint64_t, V, NUM>(A, B, sw, mw, ntiles, cbits, Crp, Ccol, Cval, s);
 }
 
 template <typename V, bool NUM>
@@ -839,12 +881,22 @@ msp_status spgemm_pass(const msp_csr *A, const msp_csr *B, const void *ws1, size
             A->nrows, A->nnz, h.nprods, A->row_offsets, sw.arow, sw.S, sw.rowlong, ntiles, mw.splits);
         st = last_launch("gemm_partition_kernel");
         if (st != MSP_OK) return st;
+        st = cuda_check(cudaMemsetAsync(&mw.totals[1], 0, 8, s), "spgemm: clear span");
+        if (st != MSP_OK) return st;
+        tile_span_kernel<<<unsigned(std::min<int64_t>(ceil_div(ntiles, 256), 148 * 4)), 256, 0, s>>>(
+            ntiles, mw.splits, sw.arow, reinterpret_cast<unsigned long long *>(&mw.totals[1]));
+        st = last_launch("tile_span_kernel");
+        if (st != MSP_OK) return st;
     } else if (m == 0 || h.nprods == 0) {
         return MSP_OK;
     }
+    int64_t maxspan = 0;  // written by the symbolic pass, kept in main_ws for numeric
+    st = cuda_check(cudaMemcpyAsync(&maxspan, &mw.totals[1], 8, cudaMemcpyDeviceToHost, s), "spgemm: span");
+    if (st == MSP_OK) st = cuda_check(cudaStreamSynchronize(s), "spgemm: sync");
+    if (st != MSP_OK) return st;
     if (h.nprods > 0) {
-        st = (A->dtype == MSP_F64) ? run_tiles<double, NUM>(A, B, sw, mw, ntiles, Crp, Ccol, Cval, s)
-                                   : run_tiles<float, NUM>(A, B, sw, mw, ntiles, Crp, Ccol, Cval, s);
+        st = (A->dtype == MSP_F64) ? run_tiles<double, NUM>(A, B, sw, mw, ntiles, maxspan, Crp, Ccol, Cval, s)
+                                   : run_tiles<float, NUM>(A, B, sw, mw, ntiles, maxspan, Crp, Ccol, Cval, s);
         if (st != MSP_OK) return st;
         st = (A->dtype == MSP_F64) ? run_long<double, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s)
                                    : run_long<float, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s);
