@@ -93,12 +93,6 @@ int msp_version(void);
 /* Diagnostics: number of libmsp kernels launched by this process so far
  * (all devices, all threads).  Used by benchmarks to report launches. */
 uint64_t msp_launch_count(void);
-/* Profiling aid: with MSP_SPMV_DEBUG=16 in the environment the SpMV kernel
- * records per-tile timestamps of its warp roles; this copies them (int64
- * ns, [CTA][tile][8]) to a HOST buffer.  Returns 0 on success, -1 if no
- * timeline was recorded, else a cudaError_t value. */
-int msp_debug_copy_timestamps(void *host, size_t bytes);
-
 /* ------------------------------------------------------------------------
  * SpMV  y = A x      (Section III-A)
  *

@@ -21,7 +21,7 @@ STATUS = {0: "MSP_OK", 1: "MSP_ERR_ARG", 2: "MSP_ERR_DTYPE", 3: "MSP_ERR_SHAPE",
 
 # every symbol include/msp.h declares (checked by tests/test_abi.py)
 EXPORTS = [
-    "msp_status_string", "msp_last_error", "msp_version", "msp_launch_count", "msp_debug_copy_timestamps",
+    "msp_status_string", "msp_last_error", "msp_version", "msp_launch_count",
     "msp_spmv_workspace", "msp_spmv",
     "msp_spadd_workspace", "msp_spadd_symbolic", "msp_spadd_numeric",
     "msp_spgemm_setup_workspace", "msp_spgemm_setup", "msp_spgemm_symbolic", "msp_spgemm_numeric",
@@ -59,7 +59,6 @@ _SIGS = {
     "msp_last_error": (ctypes.c_char_p, []),
     "msp_version": (ctypes.c_int, []),
     "msp_launch_count": (ctypes.c_uint64, []),
-    "msp_debug_copy_timestamps": (ctypes.c_int, [_vp, _sz]),
     "msp_spmv_workspace": (ctypes.c_int, [_csr_p, _P(_sz)]),
     "msp_spmv": (ctypes.c_int, [_csr_p, _vp, _vp, _vp, _sz, _vp]),
     "msp_spadd_workspace": (ctypes.c_int, [_csr_p, _csr_p, _P(_sz)]),

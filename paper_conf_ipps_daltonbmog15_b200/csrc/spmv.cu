@@ -68,7 +68,7 @@ struct Cfg {
     static constexpr int STAGES = STAGES_;
     static constexpr int MINB = MINB_;
     static constexpr int THREADS = (NW + 2) * 32;
-    static constexpr int RING = STAGES_ + RSLOTS_ + 3;   // per-tile carry slots (> max warp skew)
+    static constexpr int RING = 8;  // per-tile carry slots (power of 2; workers are in lockstep, skew <= 2 tiles)
     static constexpr int DATA_BYTES = int(((4 + sizeof(V)) * T + 64 + 15) / 16 * 16);  // rp, col, val windows
     static constexpr int FLAG_BYTES = T / 8;             // row-end bit per position
     static constexpr int RMAP_BYTES = T * 2;             // row (tile-relative, +1) ending at a position
@@ -79,13 +79,6 @@ struct Cfg {
     static constexpr int MISC_BYTES = 2048;
     static constexpr int SMEM = STAGES * STAGE_BYTES + RSLOTS * RSLOT_BYTES + PROD_BYTES + MISC_BYTES;
 };
-
-__device__ __forceinline__ uint64_t gtimer()
-{
-    uint64_t t;
-    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
-    return t;
-}
 
 __device__ __forceinline__ int ld_volatile_s(const int *p) { return *reinterpret_cast<const volatile int *>(p); }
 __device__ __forceinline__ void st_volatile_s(int *p, int v) { *reinterpret_cast<volatile int *>(p) = v; }
@@ -170,7 +163,7 @@ template <typename V, class C>
 __global__ void __launch_bounds__(C::THREADS, C::MINB)
 spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const int32_t *__restrict__ col,
                   const V *__restrict__ val, const V *__restrict__ x, V *__restrict__ y, int32_t n_cols,
-                  CtaRecord *__restrict__ recs, unsigned *__restrict__ counter, int dbg_mode, void *dbg_ts)
+                  CtaRecord *__restrict__ recs, unsigned *__restrict__ counter)
 {
     constexpr int K = C::K, NW = C::NW, WSPAN = C::WSPAN, RING = C::RING;
     constexpr int FW = C::T / 32;  // flag words per tile
@@ -238,13 +231,11 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
         }
         for (int t = 0; t < ntiles; ++t) {
             const int stage = t % C::STAGES;
-            if ((dbg_mode & 16) && lane == 0 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 0] = gtimer();
             const int64_t de = min64(d_begin + int64_t(t + 1) * C::T, d_end);
             const int lo = int(max64(i_s, de - nnz));
             const int hi = int(min64(m, de - j_s));
             const int i_e = warp_grid_search_guess(rp, de, lo, hi, i_s + prev_rows, lane);
             const int j_e = int(de - i_e);
-            if ((dbg_mode & 16) && lane == 0 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 1] = gtimer();
             prev_rows = i_e - i_s;
             if (lane == 0) {  // keep the data two tiles ahead streaming into L2
                 const int64_t rr = max(prev_rows, 32);
@@ -253,7 +244,6 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                 prefetch_range<int(sizeof(V))>(val, int64_t(j_e) + C::T, min64(j_cta_end, int64_t(j_e) + 2 * C::T));
             }
             if (t >= C::STAGES) mbar_wait_backoff(&empty[stage], ((t / C::STAGES) - 1) & 1);
-            if ((dbg_mode & 16) && lane == 0 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 2] = gtimer();
             char *sb = stages + size_t(stage) * C::STAGE_BYTES;
             const int wr_end = min(i_e + 1, m);
             // windows: rp[i_s .. wr_end] (inclusive), col/val[j_s .. j_e)
@@ -304,7 +294,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             const int z = mt.j_e - mt.j_s, i_s = mt.i_s, j_s = mt.j_s;
             for (int i = lane; i < FW; i += 32) flags[i] = 0u;
             __syncwarp();
-            if ((dbg_mode & 3) != 1) {
+            {
                 for (int r = i_s + lane; r < mt.wr_end; r += 32) {
                     const int a = rps[r - i_s] - j_s;
                     const int b = rps[r - i_s + 1] - j_s;
@@ -321,7 +311,6 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             }
             __syncwarp();
             if (lane == 0) {
-                if ((dbg_mode & 16) && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 3] = gtimer();
                 mbar_arrive(&rowsrdy[rs]);
                 mbar_arrive(&empty[stage]);  // this warp no longer reads the stage
             }
@@ -351,7 +340,6 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
         auto a_issue = [&](int t) {
             const int stage = t % C::STAGES;
             mbar_wait(&full[stage], (t / C::STAGES) & 1);
-            if ((dbg_mode & 16) && lane == 0 && warp == 0 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 6] = gtimer();
             nx_is = meta[stage].i_s;
             nx_z = meta[stage].j_e - meta[stage].j_s;
             const char *sb = stages + size_t(stage) * C::STAGE_BYTES;
@@ -368,7 +356,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             for (int u = 0; u < K; ++u) vv[u] = vs[lane + 32 * u];
         };
         auto finish_first = [&](int r, double v0, int tt) {
-            const int sl = tt % RING;
+            const int sl = tt & (RING - 1);
             double c = 0.0;
             int f = 0;
             for (int w2 = warp - 1; w2 >= 0 && !f; --w2) {
@@ -378,7 +366,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                 f = reinterpret_cast<volatile int *>(agg_f)[sl * NW + w2];
             }
             if (!f && tt > 0) {
-                const int ps = (tt - 1) % RING;
+                const int ps = (tt - 1) & (RING - 1);
                 while (ld_volatile_s(&cta_seq[ps]) != tt) {}
                 __threadfence_block();
                 c = reinterpret_cast<volatile double *>(cta_v)[ps] + c;
@@ -396,7 +384,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
         a_issue(0);
         for (int t = 0; t < ntiles; ++t) {
             const int stage = t % C::STAGES;
-            const int slot = t % RING;
+            const int slot = t & (RING - 1);
             const int rs = t % C::RSLOTS;
             const int tile_is = nx_is, z = nx_z;
             // ---- phase A finish: products -> warp-private buffer ----
@@ -406,15 +394,11 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             // the stage is released once the products are formed (releasing it
             // right after the col/val loads measured slower: deeper TMA
             // run-ahead raised memory contention and per-CTA tail variance)
+            // workers in lockstep: a warp that runs ahead would take issue slots from
+            // the slowest one, whose lag then eats the ring's slack (measured)
+            named_bar_sync(1, NW * 32);
             if (lane == 0) mbar_arrive(&empty[stage]);
-            if ((dbg_mode & 16) && lane == 0 && warp == 0 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 4] = gtimer();
             mbar_wait(&rowsrdy[rs], (t / C::RSLOTS) & 1);
-            if ((dbg_mode & 16) && lane == 0 && warp == 0 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 7] = gtimer();
-            if ((dbg_mode & 3) == 2) {  // profiling aid: phase A only
-                if (lane == 0) mbar_arrive(&rowsfree[rs]);
-                if (t + 1 < ntiles) a_issue(t + 1);
-                continue;
-            }
             // ---- walk ----
             const uint32_t *flags = reinterpret_cast<const uint32_t *>(rslots + size_t(rs) * C::RSLOT_BYTES);
             const uint16_t *rmap =
@@ -480,7 +464,6 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&rowsfree[rs]);  // done with this tile's row map
-            if ((dbg_mode & 16) && lane == 0 && warp == NW - 1 && t < 30) reinterpret_cast<uint64_t *>(dbg_ts)[blockIdx.x * 256 + t * 8 + 5] = gtimer();
             // ---- publish this warp's trailing sum; the last warp of the tile
             //      forms the carry leaving the tile ----
             if (lane == 31) {
@@ -494,7 +477,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                     double c = 0.0;
                     int f = 0;
                     if (t > 0) {
-                        const int ps = (t - 1) % RING;
+                        const int ps = (t - 1) & (RING - 1);
                         while (ld_volatile_s(&cta_seq[ps]) != t) {}
                         __threadfence_block();
                         c = cta_v[ps];
@@ -529,7 +512,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
     if (tid == 0) {
         CtaRecord rec;
         rec.carry_key = s_carry_key;
-        rec.carry_val = (ntiles > 0 && (dbg_mode & 3) == 0) ? cta_v[(ntiles - 1) % RING] : 0.0;
+        rec.carry_val = ntiles > 0 ? cta_v[(ntiles - 1) & (RING - 1)] : 0.0;
         rec.head_row = s_head_row;
         rec.head_val = s_head_val;
         recs[blockIdx.x] = rec;
@@ -571,40 +554,6 @@ template <typename V> struct Shape<V, 3> { using C = Cfg<V, 8, 2, 4, 2>; };
 template <typename V> struct Shape<V, 4> { using C = Cfg<V, 4, 2, 4, 4>; };
 constexpr int kNumShapes = 5;
 
-int debug_mode();
-int tiles_per_cta()
-{
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("MSP_SPMV_TPC");
-        v = e ? atoi(e) : (1 << 30);  // default: one persistent wave
-        if (v < 2) v = 2;
-    }
-    return v;
-}
-void *g_dbg_ts = nullptr;
-}  // namespace
-void *g_dbg_ts_public() { return g_dbg_ts; }
-namespace {
-void *debug_ts()
-{
-    if (!g_dbg_ts && (debug_mode() & 16)) {
-        cudaMalloc(&g_dbg_ts, size_t(8192) * 256 * 8);  // profiling aid only
-        cudaMemset(g_dbg_ts, 0, size_t(8192) * 256 * 8);
-    }
-    return g_dbg_ts;
-}
-
-int debug_mode()
-{
-    static int d = -1;
-    if (d < 0) {
-        const char *e = getenv("MSP_SPMV_DEBUG");
-        d = e ? atoi(e) : 0;
-    }
-    return d;
-}
-
 template <typename V, class C>
 msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
 {
@@ -631,12 +580,9 @@ msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t
         return cuda_check(cudaMemsetAsync(y, 0, size_t(A->nrows) * sizeof(V), s), "spmv: zero y");
     const int64_t total = int64_t(A->nrows) + A->nnz;
     const int64_t ntiles = ceil_div(total, C::T);
-    // Several waves of CTAs, each owning a contiguous range of about
-    // kTilesPerCta tiles: the hardware scheduler then balances CTAs that run
-    // slower than others, and a CTA's start-up search overlaps other CTAs.
-    const int64_t resident = int64_t(occ) * sm_count();
-    int64_t g = ceil_div(ntiles, tiles_per_cta());
-    if (g < resident) g = resident < ntiles ? resident : ntiles;
+    // one persistent wave, no more CTAs than tiles
+    int64_t g = int64_t(occ) * sm_count();
+    if (g > ntiles) g = ntiles;
     const int grid = int(g);
     Carve cv(ws, ws_bytes);
     unsigned *counter = cv.take<unsigned>(1);
@@ -644,7 +590,7 @@ msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t
     if (!cv.ok()) return MSP_ERR_WORKSPACE;
     kern<<<grid, C::THREADS, C::SMEM, s>>>(A->nrows, A->nnz, A->row_offsets, A->col_idx,
                                            static_cast<const V *>(A->vals), static_cast<const V *>(x),
-                                           static_cast<V *>(y), A->ncols, recs, counter, debug_mode(), debug_ts());
+                                           static_cast<V *>(y), A->ncols, recs, counter);
     return last_launch("spmv_merge_kernel");
 }
 
@@ -689,10 +635,3 @@ msp_status spmv_run(const msp_csr *A, const void *x, void *y, void *ws, size_t w
 
 }  // namespace msp
 
-// profiling aid (MSP_SPMV_DEBUG & 16): device buffer of per-tile timestamps
-extern "C" int msp_debug_copy_timestamps(void *host, size_t bytes)
-{
-    void *d = msp::g_dbg_ts_public();
-    if (!d) return -1;
-    return int(cudaMemcpy(host, d, bytes, cudaMemcpyDeviceToHost));
-}
