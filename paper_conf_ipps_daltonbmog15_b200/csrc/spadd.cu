@@ -103,26 +103,68 @@ __global__ void spadd_partition_kernel(int32_t m, int64_t nnzA, int64_t nnzB, co
 
 // --------------------------------------------------------------- tile kernel
 
+// Shared-memory layout of one tile (one CTA per tile).  The int windows
+// (A.rp, B.rp, A.col, B.col slices) and the value windows (A.val, B.val) are
+// staged by TMA bulk copies; rows + nnzA + nnzB <= T items per tile bounds
+// their total size.  Fill also stages its output run (col, val) so that C is
+// written with coalesced stores.
 template <typename V, bool FILL>
-struct AddSmem {
-    int32_t acol[ADD_T + 2];
-    int32_t bcol[ADD_T + 2];
-    int32_t arp[ADD_T + 4];
-    int32_t brp[ADD_T + 4];
-    Split st[ADD_NT + 1];
-    int32_t wsum[ADD_NT / 32];
+struct AddLayout {
+    static constexpr int IBYTES = 4 * (2 * ADD_T + 8) + 4 * 32;        // 4 int windows (+alignment slack)
+    static constexpr int VBYTES = FILL ? int(sizeof(V)) * ADD_T + 2 * 32 : 0;
+    static constexpr int OBYTES = FILL ? (4 + int(sizeof(V))) * ADD_T : 0;
+    static constexpr int V_OFF = IBYTES;
+    static constexpr int O_OFF = V_OFF + VBYTES;
+    static constexpr int ST_OFF = (O_OFF + OBYTES + 15) / 16 * 16;
+    static constexpr int WS_OFF = ST_OFF + int(sizeof(Split)) * (ADD_NT + 1);
+    static constexpr int BAR_OFF = (WS_OFF + 4 * (ADD_NT / 32) + 15) / 16 * 16;
+    static constexpr int BYTES = BAR_OFF + 16;
 };
+
+// One staged window: elements [lo, hi) of an array of `len` elements, placed
+// at a 16-byte aligned shared-memory offset; `first` = byte offset of lo.
+struct Staged {
+    WindowCopy w;
+    int off;
+};
+
+template <typename T>
+__device__ __forceinline__ Staged plan_stage(const T *base, int64_t lo, int64_t hi, int64_t len, int *off,
+                                             uint32_t *tx)
+{
+    Staged st;
+    st.w = plan_window<int(sizeof(T))>(base, lo, hi, len);
+    st.off = *off;
+    *off += int(st.w.span);
+    *tx += st.w.bulk_bytes;
+    return st;
+}
+
+// Thread 0 issues the bulk copy (after the barrier's expect_tx), lanes of
+// warp 0 copy the ragged ends; returns a pointer to element lo.
+template <typename T>
+__device__ __forceinline__ T *issue_stage(const Staged &st, const T *base, int64_t lo, int64_t hi, char *smem,
+                                          uint64_t *bar, uint64_t pol)
+{
+    char *dst = smem + st.off;
+    if (threadIdx.x == 0 && st.w.bulk_bytes) bulk_g2s(dst + st.w.bulk_dst, st.w.bulk_src, st.w.bulk_bytes, bar, pol);
+    if (threadIdx.x < 32) window_manual<T>(st.w, base, lo, hi, dst, threadIdx.x);
+    return reinterpret_cast<T *>(dst + st.w.first);
+}
 
 template <typename V, bool FILL>
 __global__ void __launch_bounds__(ADD_NT)
 spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
                   const V *__restrict__ Aval, const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
-                  const V *__restrict__ Bval, const Split *__restrict__ splits, int32_t *__restrict__ tile_count,
-                  const int64_t *__restrict__ tile_off, int32_t *__restrict__ Crp_counts, int32_t *__restrict__ Ccol,
-                  V *__restrict__ Cval)
+                  const V *__restrict__ Bval, int64_t nnzA, int64_t nnzB, const Split *__restrict__ splits,
+                  int32_t *__restrict__ tile_count, const int64_t *__restrict__ tile_off,
+                  int32_t *__restrict__ Crp_counts, int32_t *__restrict__ Ccol, V *__restrict__ Cval)
 {
-    extern __shared__ __align__(16) char smem_raw[];
-    AddSmem<V, FILL> &S = *reinterpret_cast<AddSmem<V, FILL> *>(smem_raw);
+    using L = AddLayout<V, FILL>;
+    extern __shared__ __align__(128) char smem_raw[];
+    Split *S_st = reinterpret_cast<Split *>(smem_raw + L::ST_OFF);
+    int32_t *S_wsum = reinterpret_cast<int32_t *>(smem_raw + L::WS_OFF);
+    uint64_t *bar = reinterpret_cast<uint64_t *>(smem_raw + L::BAR_OFF);
     const int tid = threadIdx.x;
     const int k = blockIdx.x;
     const Split s0 = splits[k], s1 = splits[k + 1];
@@ -130,35 +172,56 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
     const int ga0 = s0.a, gb0 = s0.b;
     const int nA = s1.a - ga0, nB = s1.b - gb0;
     const int nrw = min(r1, m - 1) - r0 + 2;  // row offsets r0 .. min(r1, m-1)+1
-    // ---- stage the tile (coalesced asynchronous copies, all in flight) ----
-    for (int i = tid; i < nA; i += ADD_NT) cp_async<4>(&S.acol[i], Acol + ga0 + i);
-    for (int i = tid; i < nB; i += ADD_NT) cp_async<4>(&S.bcol[i], Bcol + gb0 + i);
-    for (int i = tid; i < nrw; i += ADD_NT) {
-        cp_async<4>(&S.arp[i], Arp + r0 + i);
-        cp_async<4>(&S.brp[i], Brp + r0 + i);
+    if (tid == 0) {
+        mbar_init(bar, 1);
+        fence_mbar_init();
     }
-    cp_async_wait_all();
     __syncthreads();
+    // ---- stage the tile: one TMA bulk copy per window ----
+    const uint64_t pol = policy_evict_first();
+    int ioff = 0, voff = L::V_OFF;
+    uint32_t tx = 0;
+    const Staged p_arp = plan_stage<int32_t>(Arp, r0, r0 + nrw, int64_t(m) + 1, &ioff, &tx);
+    const Staged p_brp = plan_stage<int32_t>(Brp, r0, r0 + nrw, int64_t(m) + 1, &ioff, &tx);
+    const Staged p_ac = plan_stage<int32_t>(Acol, ga0, ga0 + nA, nnzA, &ioff, &tx);
+    const Staged p_bc = plan_stage<int32_t>(Bcol, gb0, gb0 + nB, nnzB, &ioff, &tx);
+    Staged p_av{}, p_bv{};
+    if constexpr (FILL) {
+        p_av = plan_stage<V>(Aval, ga0, ga0 + nA, nnzA, &voff, &tx);
+        p_bv = plan_stage<V>(Bval, gb0, gb0 + nB, nnzB, &voff, &tx);
+    }
+    if (tid == 0) mbar_arrive_expect_tx(bar, tx);
+    int32_t *arp = issue_stage<int32_t>(p_arp, Arp, r0, r0 + nrw, smem_raw, bar, 0);
+    int32_t *brp = issue_stage<int32_t>(p_brp, Brp, r0, r0 + nrw, smem_raw, bar, 0);
+    const int32_t *acs = issue_stage<int32_t>(p_ac, Acol, ga0, ga0 + nA, smem_raw, bar, pol);
+    const int32_t *bcs = issue_stage<int32_t>(p_bc, Bcol, gb0, gb0 + nB, smem_raw, bar, pol);
+    const V *avs = nullptr, *bvs = nullptr;
+    if constexpr (FILL) {
+        avs = issue_stage<V>(p_av, Aval, ga0, ga0 + nA, smem_raw, bar, pol);
+        bvs = issue_stage<V>(p_bv, Bval, gb0, gb0 + nB, smem_raw, bar, pol);
+    }
+    mbar_wait(bar, 0);
+    __syncthreads();  // ragged ends written by warp 0
     for (int i = tid; i < nrw; i += ADD_NT) {  // tile-relative row offsets
-        S.arp[i] -= ga0;
-        S.brp[i] -= gb0;
+        arp[i] -= ga0;
+        brp[i] -= gb0;
     }
     __syncthreads();
     const int nrows = r1 - r0;  // row-end items in the tile
     const int items = nrows + nA + nB;
-    auto a_lo = [&](int r) { return max(S.arp[r - r0], 0); };
-    auto a_hi = [&](int r) { return min(S.arp[r - r0 + 1], nA); };
-    auto b_lo = [&](int r) { return max(S.brp[r - r0], 0); };
-    auto b_hi = [&](int r) { return min(S.brp[r - r0 + 1], nB); };
-    auto acol = [&](int i) { return S.acol[i]; };
-    auto bcol = [&](int i) { return S.bcol[i]; };
+    auto a_lo = [&](int r) { return max(arp[r - r0], 0); };
+    auto a_hi = [&](int r) { return min(arp[r - r0 + 1], nA); };
+    auto b_lo = [&](int r) { return max(brp[r - r0], 0); };
+    auto b_hi = [&](int r) { return min(brp[r - r0 + 1], nB); };
+    auto acol = [&](int i) { return acs[i]; };
+    auto bcol = [&](int i) { return bcs[i]; };
     // ---- this thread's split ----
     {
         const int dt = min(tid * ADD_IPT, items);
         int lo = max(0, dt - (nA + nB)), hi = min(dt, nrows);
         while (lo < hi) {
             const int mid = (lo + hi) >> 1;
-            const int rend = min(S.arp[mid + 1], nA) + min(S.brp[mid + 1], nB);
+            const int rend = min(arp[mid + 1], nA) + min(brp[mid + 1], nB);
             if (rend <= dt - mid - 1) lo = mid + 1;
             else hi = mid;
         }
@@ -173,15 +236,15 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
             const int al = a_lo(r), ah = a_hi(r), bl = b_lo(r), bh = b_hi(r);
             int ia, ib;
             row_merge_path(acol, al, ah, bcol, bl, bh, e - (al + bl), ia, ib);
-            if (ia > al && ib < bh && S.acol[ia - 1] == S.bcol[ib]) ++ib;  // balanced path
+            if (ia > al && ib < bh && acs[ia - 1] == bcs[ib]) ++ib;  // balanced path
             st.a = ia;
             st.b = ib;
         }
-        S.st[tid] = st;
-        if (tid == 0) S.st[ADD_NT] = Split{r1, nA, nB};
+        S_st[tid] = st;
+        if (tid == 0) S_st[ADD_NT] = Split{r1, nA, nB};
     }
     __syncthreads();
-    const Split beg = S.st[tid], end = S.st[tid + 1];
+    const Split beg = S_st[tid], end = S_st[tid + 1];
 
     // ---- walk: Alg. 1 order; row-end items close rows ----
     auto walk = [&](auto &&on_out, auto &&on_row_end) {
@@ -198,24 +261,25 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
                 }
                 continue;
             }
-            if (ra && (!rb || S.acol[ia] <= S.bcol[ib])) {
-                if (rb && S.acol[ia] == S.bcol[ib]) {
-                    on_out(S.acol[ia], ia, ib);
+            const int ca = ra ? acs[ia] : INT_MAX, cb = rb ? bcs[ib] : INT_MAX;
+            if (ca <= cb) {
+                if (ca == cb) {
+                    on_out(ca, ia, ib);
                     ++ia;
                     ++ib;
                 } else {
-                    on_out(S.acol[ia], ia, -1);
+                    on_out(ca, ia, -1);
                     ++ia;
                 }
             } else {
-                on_out(S.bcol[ib], -1, ib);
+                on_out(cb, -1, ib);
                 ++ib;
             }
         }
         return r;
     };
 
-    if (!FILL) {
+    if constexpr (!FILL) {
         int cnt = 0, total = 0;
         const int r_last = walk([&](int, int, int) { ++cnt; ++total; },
                                 [&](int r) {
@@ -227,33 +291,37 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
         int wsum = total;
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) wsum += __shfl_xor_sync(0xffffffffu, wsum, o);
-        if ((tid & 31) == 0) S.wsum[tid >> 5] = wsum;
+        if ((tid & 31) == 0) S_wsum[tid >> 5] = wsum;
         __syncthreads();
         if (tid == 0) {
             int t = 0;
-            for (int w = 0; w < ADD_NT / 32; ++w) t += S.wsum[w];
+            for (int w = 0; w < ADD_NT / 32; ++w) t += S_wsum[w];
             tile_count[k] = t;
         }
     } else {
+        int32_t *ocol = reinterpret_cast<int32_t *>(smem_raw + L::O_OFF);
+        V *oval = reinterpret_cast<V *>(smem_raw + L::O_OFF + 4 * ADD_T);
         int cnt = 0;
         walk([&](int, int, int) { ++cnt; }, [&](int) {});
         int tot;
-        const int off = block_exclusive_sum<int, ADD_NT / 32>(cnt, S.wsum, 0, &tot);
-        // outputs of this thread are consecutive in C: store them directly
-        // (values read from global at the matched positions, L1-resident)
-        const int64_t base = tile_off[k] + off;
-        int o = 0;
+        int o = block_exclusive_sum<int, ADD_NT / 32>(cnt, S_wsum, 0, &tot);
         walk(
             [&](int c, int ia, int ib) {
                 V v;
-                if (ia >= 0 && ib >= 0) v = Aval[ga0 + ia] + Bval[gb0 + ib];  // one rounding, A first
-                else v = (ia >= 0) ? Aval[ga0 + ia] : Bval[gb0 + ib];
-                Ccol[base + o] = c;
-                Cval[base + o] = v;
+                if (ia >= 0 && ib >= 0) v = avs[ia] + bvs[ib];  // one rounding, A first (Alg. 1)
+                else v = (ia >= 0) ? avs[ia] : bvs[ib];
+                ocol[o] = c;
+                oval[o] = v;
                 ++o;
             },
             [&](int) {});
-        (void)tot;
+        __syncthreads();
+        // the tile's run of C is contiguous: coalesced stores
+        const int64_t base = tile_off[k];
+        for (int i = tid; i < tot; i += ADD_NT) {
+            Ccol[base + i] = ocol[i];
+            Cval[base + i] = oval[i];
+        }
     }
 }
 
@@ -290,7 +358,7 @@ msp_status launch_tiles(const msp_csr *A, const msp_csr *B, const AddWs &w, int3
                         cudaStream_t s)
 {
     auto kern = spadd_tile_kernel<V, FILL>;
-    const int smem = int(sizeof(AddSmem<V, FILL>));
+    const int smem = AddLayout<V, FILL>::BYTES;
     static int configured = 0;
     if (!configured) {
         msp_status st = cuda_check(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem),
@@ -300,7 +368,7 @@ msp_status launch_tiles(const msp_csr *A, const msp_csr *B, const AddWs &w, int3
     }
     kern<<<unsigned(w.ntiles), ADD_NT, smem, s>>>(
         A->nrows, A->row_offsets, A->col_idx, static_cast<const V *>(A->vals), B->row_offsets, B->col_idx,
-        static_cast<const V *>(B->vals), w.splits, w.tile_count, w.tile_off, Crp ? Crp + 1 : nullptr, Ccol,
+        static_cast<const V *>(B->vals), A->nnz, B->nnz, w.splits, w.tile_count, w.tile_off, Crp ? Crp + 1 : nullptr, Ccol,
         static_cast<V *>(Cval));
     return last_launch(FILL ? "spadd_tile_kernel<fill>" : "spadd_tile_kernel<count>");
 }

@@ -33,6 +33,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <algorithm>
+#include <cmath>
 #include <type_traits>
 
 #include "common.cuh"
@@ -61,6 +62,7 @@ struct CtaRecord {  // one per CTA in the workspace
 // merge items), plus one producer warp and one row warp.
 template <typename V, int NW_, int STAGES_, int RSLOTS_, int MINB_>
 struct Cfg {
+    static constexpr bool ROWK = false;
     static constexpr int NW = NW_;
     static constexpr int K = 8;
     static constexpr int WSPAN = 32 * K;                 // products per worker warp
@@ -70,7 +72,8 @@ struct Cfg {
     static constexpr int THREADS = (NW + 2) * 32;
     static constexpr int RING = 8;  // per-tile carry slots (power of 2; workers are in lockstep, skew <= 2 tiles)
     static constexpr int DATA_BYTES = int(((4 + sizeof(V)) * T + 64 + 15) / 16 * 16);  // rp, col, val windows
-    static constexpr int FLAG_BYTES = T / 8;             // row-end bit per position
+    static constexpr int FW = T / 32;                    // flag words per tile
+    static constexpr int FLAG_BYTES = FW * 4;            // row-end bit per position
     static constexpr int RMAP_BYTES = T * 2;             // row (tile-relative, +1) ending at a position
     static constexpr int STAGE_BYTES = DATA_BYTES;       // TMA ring: released after phase A
     static constexpr int RSLOTS = RSLOTS_;               // row-map ring: released after the walk
@@ -78,6 +81,37 @@ struct Cfg {
     static constexpr int PROD_BYTES = NW * WSPAN * 8;    // warp-private product buffers
     static constexpr int MISC_BYTES = 2048;
     static constexpr int SMEM = STAGES * STAGE_BYTES + RSLOTS * RSLOT_BYTES + PROD_BYTES + MISC_BYTES;
+};
+
+// Row-aligned variant (reading R2): every lane owns K
+// consecutive products of the tile, K chosen per matrix from its mean row
+// length (odd, so the lane-strided shared-memory reads of col/val are bank
+// conflict free).  The products stay in registers (no transpose buffer), and
+// when rows are about K long, gather u of the 32 lanes touches the same
+// stencil position of 32 consecutive rows -- a few x cache lines per
+// instruction instead of one per row.
+template <typename V, int NW_, int K_, int STAGES_, int MINB_>
+struct CfgK {
+    static constexpr bool ROWK = true;
+    static constexpr int NW = NW_;
+    static constexpr int K = K_;
+    static constexpr int WSPAN = 32 * K;
+    static constexpr int T = NW * WSPAN;
+    static constexpr int STAGES = STAGES_;
+    static constexpr int MINB = MINB_;
+    static constexpr int THREADS = (NW + 2) * 32;
+    static constexpr int RING = 8;
+    static constexpr int DATA_BYTES = int(((4 + sizeof(V)) * T + 64 + 15) / 16 * 16);
+    static constexpr int FW = (T + 31) / 32 + 1;         // +1: lane masks read two words
+    static constexpr int FLAG_BYTES = (FW * 4 + 15) / 16 * 16;
+    static constexpr int RMAP_BYTES = (T * 2 + 15) / 16 * 16;
+    static constexpr int STAGE_BYTES = DATA_BYTES;
+    static constexpr int RSLOTS = STAGES_;
+    static constexpr int RSLOT_BYTES = FLAG_BYTES + RMAP_BYTES;
+    static constexpr int PROD_BYTES = 0;
+    static constexpr int MISC_BYTES = 2048;
+    static constexpr int SMEM = STAGES * STAGE_BYTES + RSLOTS * RSLOT_BYTES + PROD_BYTES + MISC_BYTES;
+    static_assert(K % 2 == 1 && K < 32, "K odd and < 32");
 };
 
 __device__ __forceinline__ int ld_volatile_s(const int *p) { return *reinterpret_cast<const volatile int *>(p); }
@@ -108,6 +142,22 @@ __device__ __forceinline__ int warp_grid_search(const int32_t *__restrict__ rp, 
     bool pred = false;
     if (p < hi) pred = int64_t(__ldg(rp + p + 1)) <= d - p - 1;
     return lo + __popc(__ballot_sync(0xffffffffu, pred));
+}
+
+// x gathers as volatile asm: issued in program order ahead of the row-map
+// wait (plain __ldg loads are sunk past it by the compiler, serialising each
+// gather's latency with the multiply-add that uses it).
+__device__ __forceinline__ double ldg_x(const double *p)
+{
+    double v;
+    asm volatile("ld.global.f64 %0, [%1];" : "=d"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ double ldg_x(const float *p)
+{
+    float v;
+    asm volatile("ld.global.f32 %0, [%1];" : "=f"(v) : "l"(p) : "memory");
+    return double(v);
 }
 
 __device__ __forceinline__ void mbar_wait_backoff(uint64_t *bar, uint32_t parity)
@@ -166,7 +216,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                   CtaRecord *__restrict__ recs, unsigned *__restrict__ counter)
 {
     constexpr int K = C::K, NW = C::NW, WSPAN = C::WSPAN, RING = C::RING;
-    constexpr int FW = C::T / 32;  // flag words per tile
+    constexpr int FW = C::FW;
     extern __shared__ __align__(128) char smem[];
     char *stages = smem;
     char *rslots = smem + C::STAGES * C::STAGE_BYTES;                   // [RSLOTS] flags + row map
@@ -295,6 +345,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             for (int i = lane; i < FW; i += 32) flags[i] = 0u;
             __syncwarp();
             {
+#pragma unroll 4
                 for (int r = i_s + lane; r < mt.wr_end; r += 32) {
                     const int a = rps[r - i_s] - j_s;
                     const int b = rps[r - i_s + 1] - j_s;
@@ -315,6 +366,138 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                 mbar_arrive(&empty[stage]);  // this warp no longer reads the stage
             }
         }
+    } else if constexpr (C::ROWK) {
+        // ===================== worker warps (row-aligned) =====================
+        // Lane l of worker `warp` owns products [q0, q0 + K), q0 = warp*32K +
+        // l*K, of every tile: it gathers their x entries (K loads in flight),
+        // then walks them in order -- fp64 multiply-add into a running sum,
+        // y written at each row end (its first row end waits for the carry of
+        // earlier lanes); the warp segmented scan and the look-back across
+        // warps / tiles are the same as in the transpose variant below.
+        const int q0 = warp * WSPAN + lane * K;
+        const int fw0 = q0 >> 5, fsh = q0 & 31;
+        auto finish_first = [&](int r, double v0, int tt) {
+            const int sl = tt & (RING - 1);
+            double c = 0.0;
+            int f = 0;
+            for (int w2 = warp - 1; w2 >= 0 && !f; --w2) {
+                while (ld_volatile_s(&agg_seq[sl * NW + w2]) != tt + 1) {}
+                __threadfence_block();
+                c = reinterpret_cast<volatile double *>(agg_v)[sl * NW + w2] + c;
+                f = reinterpret_cast<volatile int *>(agg_f)[sl * NW + w2];
+            }
+            if (!f && tt > 0) {
+                const int ps = (tt - 1) & (RING - 1);
+                while (ld_volatile_s(&cta_seq[ps]) != tt) {}
+                __threadfence_block();
+                c = reinterpret_cast<volatile double *>(cta_v)[ps] + c;
+                f = reinterpret_cast<volatile int *>(cta_f)[ps];
+            }
+            const double v = v0 + c;
+            y[r] = V(v);
+            if (!f) {
+                s_head_row = r;
+                s_head_val = v;
+            }
+        };
+        int pend_r = -1, pend_t = 0;
+        double pend_v = 0.0;
+        for (int t = 0; t < ntiles; ++t) {
+            const int stage = t % C::STAGES;
+            const int slot = t & (RING - 1);
+            const int rs = t % C::RSLOTS;
+            mbar_wait(&full[stage], (t / C::STAGES) & 1);
+            const int tile_is = meta[stage].i_s;
+            const int z = meta[stage].j_e - meta[stage].j_s;
+            const char *sb = stages + size_t(stage) * C::STAGE_BYTES;
+            const int32_t *cs = reinterpret_cast<const int32_t *>(sb + meta[stage].col_first);
+            const V *vs = reinterpret_cast<const V *>(sb + meta[stage].val_first);
+            // ---- gathers: K independent loads in flight per lane ----
+            double xv[K];
+#pragma unroll
+            for (int u = 0; u < K; ++u) {
+                const int q = q0 + u;
+                xv[u] = 0.0;
+                if (q < z) xv[u] = ldg_x(x + cs[q]);
+            }
+            mbar_wait(&rowsrdy[rs], (t / C::RSLOTS) & 1);
+            const uint32_t *flags = reinterpret_cast<const uint32_t *>(rslots + size_t(rs) * C::RSLOT_BYTES);
+            const uint16_t *rmap =
+                reinterpret_cast<const uint16_t *>(rslots + size_t(rs) * C::RSLOT_BYTES + C::FLAG_BYTES);
+            const unsigned mask = __funnelshift_r(flags[fw0], flags[fw0 + 1], fsh) & ((1u << K) - 1u);
+            // ---- walk ----
+            double run = 0.0, first_v = 0.0;
+            int first_k = -1;
+#pragma unroll
+            for (int u = 0; u < K; ++u) {
+                const int q = q0 + u;
+                if (q < z) run = fma(double(vs[q]), xv[u], run);
+                if ((mask >> u) & 1u) {
+                    if (first_k < 0) {
+                        first_k = u;
+                        first_v = run;
+                    } else {
+                        y[tile_is + int(rmap[q]) - 1] = V(run);
+                    }
+                    run = 0.0;
+                }
+            }
+            const int first_r = first_k >= 0 ? tile_is + int(rmap[q0 + first_k]) - 1 : -1;
+            __syncwarp();
+            if (lane == 0) {  // stage and row map of this tile no longer read by this warp
+                mbar_arrive(&empty[stage]);
+                mbar_arrive(&rowsfree[rs]);
+            }
+            const bool flagged = first_r >= 0;
+            // ---- warp segmented scan ----
+            const SegPair<double> inc = warp_seg_inclusive(SegPair<double>{flagged, run}, lane);
+            const double exv = __shfl_up_sync(0xffffffffu, inc.v, 1);
+            const unsigned fmask = __ballot_sync(0xffffffffu, flagged);
+            const int flane = fmask ? __ffs(fmask) - 1 : 32;
+            double pend_nv = 0.0;
+            if (flagged) {
+                const double v = lane ? first_v + exv : first_v;
+                if (lane == flane) pend_nv = v;
+                else y[first_r] = V(v);
+            }
+            // ---- publish the warp's trailing sum; the last warp forms the
+            //      carry leaving the tile ----
+            if (lane == 31) {
+                agg_v[slot * NW + warp] = inc.v;
+                agg_f[slot * NW + warp] = inc.f;
+                __threadfence_block();
+                st_volatile_s(&agg_seq[slot * NW + warp], t + 1);
+                const int done = atomicAdd(&pub_cnt[slot], 1);
+                if (done == NW - 1) {
+                    __threadfence_block();
+                    double c = 0.0;
+                    int f = 0;
+                    if (t > 0) {
+                        const int ps = (t - 1) & (RING - 1);
+                        while (ld_volatile_s(&cta_seq[ps]) != t) {}
+                        __threadfence_block();
+                        c = cta_v[ps];
+                        f = cta_f[ps];
+                    }
+                    for (int w2 = 0; w2 < NW; ++w2) {
+                        const int fw = reinterpret_cast<volatile int *>(agg_f)[slot * NW + w2];
+                        const double vw = reinterpret_cast<volatile double *>(agg_v)[slot * NW + w2];
+                        c = fw ? vw : c + vw;
+                        f |= fw;
+                    }
+                    cta_v[slot] = c;
+                    cta_f[slot] = f;
+                    pub_cnt[slot] = 0;
+                    __threadfence_block();
+                    st_volatile_s(&cta_seq[slot], t + 1);
+                }
+            }
+            if (pend_r >= 0) finish_first(pend_r, pend_v, pend_t);
+            pend_r = (lane == flane) ? first_r : -1;
+            pend_v = pend_nv;
+            pend_t = t;
+        }
+        if (pend_r >= 0) finish_first(pend_r, pend_v, pend_t);
     } else {
         // ============================ worker warps =============================
         // Worker `warp` owns products [warp*256, warp*256 + 256) of every tile.
@@ -569,7 +752,9 @@ msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t
         if (st != MSP_OK) return st;
         st = cuda_check(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, C::THREADS, C::SMEM),
                         "spmv: occupancy");
-        if (getenv("MSP_VERBOSE")) fprintf(stderr, "msp spmv: T=%d stages=%d smem=%d occupancy=%d CTAs/SM\n", C::T, C::STAGES, C::SMEM, occ);
+        if (getenv("MSP_VERBOSE"))
+            fprintf(stderr, "msp spmv: rowk=%d K=%d NW=%d T=%d stages=%d smem=%d occupancy=%d CTAs/SM\n", int(C::ROWK), C::K,
+                    C::NW, C::T, C::STAGES, C::SMEM, occ);
         if (st != MSP_OK) return st;
         if (occ < 1) occ = 1;
         if (occ > 4) occ = 4;
@@ -596,19 +781,63 @@ msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t
 
 int shape_choice()
 {
-    static int c = -1;
-    if (c < 0) {
+    static int c = -2;
+    if (c == -2) {
         const char *e = getenv("MSP_SPMV_CFG");
-        c = e ? atoi(e) : 0;
-        if (c < 0 || c >= kNumShapes) c = 0;
+        c = e ? atoi(e) : -1;  // -1: row-aligned variant (default)
+        if (c < -1 || c >= kNumShapes) c = -1;
     }
     return c;
+}
+
+// Row-aligned variant: K = the instantiated odd width nearest the mean row
+// length (MSP_SPMV_K overrides, tuning only); NW worker warps per CTA.
+constexpr int kKs[] = {7, 11, 15, 19, 23, 27, 31};
+
+int k_choice(const msp_csr *A)
+{
+    const char *e = getenv("MSP_SPMV_K");
+    const double avg = e ? atof(e) : (A->nrows > 0 ? double(A->nnz) / double(A->nrows) : 0.0);
+    int best = kKs[0];
+    for (int k : kKs)
+        if (std::abs(double(k) - avg) < std::abs(double(best) - avg)) best = k;
+    return best;
+}
+
+int nw_choice()
+{
+    static int nw = -1;
+    if (nw < 0) {
+        const char *e = getenv("MSP_SPMV_NW");
+        nw = (e && atoi(e) == 4) ? 4 : 8;
+    }
+    return nw;
+}
+
+template <typename V, int NW>
+msp_status launch_k(int K, const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
+{
+    constexpr int MB = NW == 4 ? 2 : 1;
+    switch (K) {
+    case 7: return launch_cfg<V, CfgK<V, NW, 7, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    case 11: return launch_cfg<V, CfgK<V, NW, 11, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    case 15: return launch_cfg<V, CfgK<V, NW, 15, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    case 19: return launch_cfg<V, CfgK<V, NW, 19, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    case 23: return launch_cfg<V, CfgK<V, NW, 23, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    case 27: return launch_cfg<V, CfgK<V, NW, 27, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    default: return launch_cfg<V, CfgK<V, NW, 31, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    }
 }
 
 template <typename V>
 msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
 {
     switch (shape_choice()) {
+    case -1: {
+        const int K = k_choice(A);
+        return nw_choice() == 8 ? launch_k<V, 8>(K, A, x, y, ws, ws_bytes, s)
+                                : launch_k<V, 4>(K, A, x, y, ws, ws_bytes, s);
+    }
     case 1: return launch_cfg<V, typename Shape<V, 1>::C>(A, x, y, ws, ws_bytes, s);
     case 2: return launch_cfg<V, typename Shape<V, 2>::C>(A, x, y, ws, ws_bytes, s);
     case 3: return launch_cfg<V, typename Shape<V, 3>::C>(A, x, y, ws, ws_bytes, s);
