@@ -200,11 +200,28 @@ def random_rows(n: int = 100_000_000, max_len: int = 8, seed: int = 5, ncols: in
     ncols = n if ncols is None else ncols
     rng = np.random.default_rng(seed)
     lens = rng.integers(0, max_len + 1, size=n).astype(np.int64)
-    rows = np.repeat(np.arange(n, dtype=np.int64), lens)
-    cols = rng.integers(0, ncols, size=rows.size, dtype=np.int64)
-    keys = np.unique(rows * ncols + cols)
-    rp, col = _from_sorted_keys(keys, n, ncols)
-    return CSR(n, ncols, rp, col, np.ones(col.size))
+    # Rows in blocks: a padded [rows, max_len] block of draws, slot k >= len
+    # masked with a sentinel, sorted along each row, adjacent duplicates
+    # dropped (vectorised; a global unique over 4e8 keys takes minutes).
+    sent = np.iinfo(np.int64).max
+    counts = np.zeros(n, dtype=np.int64)
+    parts = []
+    blk = 1 << 22
+    for s in range(0, n, blk):
+        e = min(n, s + blk)
+        c = rng.integers(0, ncols, size=(e - s, max_len), dtype=np.int64)
+        c[np.arange(max_len)[None, :] >= lens[s:e, None]] = sent
+        c.sort(axis=1)
+        keep = c != sent
+        keep[:, 1:] &= c[:, 1:] != c[:, :-1]
+        counts[s:e] = keep.sum(axis=1)
+        parts.append(c[keep].astype(np.int32))
+    rp = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(counts, out=rp[1:])
+    if rp[-1] > np.iinfo(np.int32).max:
+        raise ValueError("nnz exceeds int32")
+    col = np.concatenate(parts) if parts else np.zeros(0, np.int32)
+    return CSR(n, ncols, rp.astype(np.int32), col, np.ones(col.size))
 
 
 def random_csr(m: int, n: int, seed: int, density: float = 0.1, empty_frac: float = 0.0,
