@@ -784,8 +784,9 @@ int shape_choice()
     static int c = -2;
     if (c == -2) {
         const char *e = getenv("MSP_SPMV_CFG");
-        c = e ? atoi(e) : -1;  // -1: row-aligned variant (default)
-        if (c < -1 || c >= kNumShapes) c = -1;
+        // -3: chosen per matrix (default), -1: row-aligned variant, 0..: transpose-walk shapes
+        c = e ? atoi(e) : -3;
+        if (c < -3 || c >= kNumShapes) c = -3;
     }
     return c;
 }
@@ -832,7 +833,10 @@ msp_status launch_k(int K, const msp_csr *A, const void *x, void *y, void *ws, s
 template <typename V>
 msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
 {
-    switch (shape_choice()) {
+    int shape = shape_choice();
+    if (shape == -3)  // default: row-aligned lanes for long regular rows, transpose walk otherwise
+        shape = (A->nrows > 0 && double(A->nnz) >= 20.0 * double(A->nrows)) ? -1 : 0;
+    switch (shape) {
     case -1: {
         const int K = k_choice(A);
         return nw_choice() == 8 ? launch_k<V, 8>(K, A, x, y, ws, ws_bytes, s)

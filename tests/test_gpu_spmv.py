@@ -125,3 +125,20 @@ def test_fp32_long_row_accumulates_in_fp64():
                 np.concatenate([[2.0 ** 24], np.ones(n - 1)]).astype(np.float32))
     y = run(A, np.ones(n, np.float32))
     assert y[0] == np.float32(2.0 ** 24 + 4096)
+
+
+@pytest.mark.parametrize("L", [3, 5, 7, 27])
+def test_cta_boundary_before_row_end(L):
+    """Uniform rows of L nonzeros: the persistent grid's diagonal split
+    b*(m+nnz)/G falls, for about one CTA in L+1, between a row's last nonzero
+    and its row-end item, so the CTA's trailing partial belongs to a row whose
+    end the next CTA consumes first (Z21: carries are (row, partial) pairs)."""
+    for m in (150_001, 200_003, 333_331):
+        n = m
+        rp = (np.arange(m + 1, dtype=np.int64) * L).astype(np.int32)
+        col = np.tile((np.arange(L) * (n // L)).astype(np.int32), m)  # sorted, distinct per row
+        val = gen.int_values(m * L, L)
+        A = gen.CSR(m, n, rp, col, val)
+        x = gen.x_vector(n, "int")
+        y = run(A, x)
+        assert np.array_equal(y, oracle.spmv(A, x)[0]), f"m={m} L={L}"

@@ -16,7 +16,7 @@ def main():
     A = gen.config(cfg, "random")
     dA = msp.CsrTensor.from_arrays(A.rp, A.col, A.val, (A.m, A.n), "cuda")
     if op == "spmv":
-        x = torch.from_numpy(gen.matrices.x_vector(A.n, "random")).cuda()
+        x = torch.from_numpy(gen.matrices.x_vector(A.n, "random", dtype=A.val.dtype)).cuda()
         for _ in range(reps):
             msp.spmv(dA, x)
     elif op == "spadd":

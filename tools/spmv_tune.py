@@ -55,7 +55,7 @@ def main():
         env = dict(os.environ)
         for kv in spec.split(","):
             k, v = kv.split("=")
-            env["MSP_SPMV_" + k] = v
+            env[k if k.startswith("MSP_") else "MSP_SPMV_" + k] = v
         env["MSP_VERBOSE"] = "1"
         r = subprocess.run([sys.executable, "-c", CHILD, cfg], env=env, capture_output=True, text=True)
         line = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
