@@ -215,13 +215,26 @@ struct TileKeys {
         BlockSortSmem<GM_NT, GM_IPT, KT> sort;
     };
 };
+template <>
+struct TileKeys<uint32_t, false> {
+    union {
+        uint32_t stage[GM_T];
+        BlockSortSmem<GM_NT, GM_IPT, uint32_t> sort;
+        RunSortSmem<GM_T, uint32_t> rm;
+    };
+};
 template <typename KT>
 struct TileKeys<KT, true> {
     KT stage[GM_T];
 };
+// symbolic with 32-bit keys: run table of the run-aware sort (64-bit keys
+// keep the generic sort: their larger state would spill at 2 CTAs/SM)
+template <typename KT, bool NUM> struct TileRuns { char t; };
+template <> struct TileRuns<uint32_t, false> { RunTable t; };
 template <typename KT, bool NUM>
 struct TileSmem {
     TileKeys<KT, NUM> keys;
+    TileRuns<KT, NUM> runs;
     double vals[NUM ? GM_T : 1];
     KT edge_first[GM_NT];
     KT edge_last[GM_NT];
@@ -271,14 +284,23 @@ __device__ __forceinline__ void sort_compress(TileSmem<KT, NUM> &Sm, int np, int
     static_assert(GM_IPT == 16 && GM_T <= 65536, "permutation packing");
     uint4 *pp = reinterpret_cast<uint4 *>(tperm + tid * GM_IPT);
     if constexpr (!NUM) {
+        // products arrive as sorted B-row runs grouped by row: merge runs
+        // within rows; the generic block sort is the fallback for tiles with
+        // very many runs
+        bool sorted = false;
+        if constexpr (sizeof(KT) == 4)
+            sorted = run_merge_sort<GM_NT, GM_IPT, KT>(Sm.keys.stage, np, Sm.keys.rm, Sm.runs.t, Sm.wsum,
+                                                       [&](KT kk) { return O::row(kk, cbits); }, k, v);
+        if (!sorted) {
 #pragma unroll
-        for (int u = 0; u < GM_IPT; ++u) {
-            const int slot = tid + u * GM_NT;
-            k[u] = slot < np ? Sm.keys.stage[slot] : O::MASKED;
-            v[u] = slot;
+            for (int u = 0; u < GM_IPT; ++u) {
+                const int slot = tid + u * GM_NT;
+                k[u] = slot < np ? Sm.keys.stage[slot] : O::MASKED;
+                v[u] = slot;
+            }
+            __syncthreads();  // staging is reused by the sort
+            block_merge_sort<GM_NT, GM_IPT, KT>(k, v, Sm.keys.sort);
         }
-        __syncthreads();  // staging is reused by the sort
-        block_merge_sort<GM_NT, GM_IPT, KT>(k, v, Sm.keys.sort);
         uint32_t w[GM_IPT / 2];
 #pragma unroll
         for (int i = 0; i < GM_IPT / 2; ++i) w[i] = uint32_t(v[2 * i]) | (uint32_t(v[2 * i + 1]) << 16);
