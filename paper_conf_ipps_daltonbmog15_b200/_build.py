@@ -23,7 +23,7 @@ BUILD = ROOT / "build" / "msp"
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
-         "--expt-relaxed-constexpr", "-I", str(ROOT / "include")]
+         "--expt-relaxed-constexpr", "-I", str(ROOT / "include")] + os.environ.get("MSP_NVCC_EXTRA", "").split()
 
 
 def sources() -> list[Path]:

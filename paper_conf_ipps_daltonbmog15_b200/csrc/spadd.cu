@@ -40,7 +40,10 @@ namespace msp {
 namespace {
 
 constexpr int ADD_NT = 256;
-constexpr int ADD_IPT = 8;
+#ifndef MSP_ADD_IPT
+#define MSP_ADD_IPT 12  // measured on B200: C3 A+A^T 1.96 ms at 8, 1.71 at 12, 1.83 at 16
+#endif
+constexpr int ADD_IPT = MSP_ADD_IPT;  // merge items per thread
 constexpr int ADD_T = ADD_NT * ADD_IPT;  // merge items per tile
 
 struct Split {
