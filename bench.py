@@ -110,6 +110,22 @@ def workload(rank: int, world: int):
     return G, None, int(starts[rank]), int(starts[rank + 1])
 
 
+def ncu_traffic(world):
+    """DRAM bytes per launch of the SpMV kernel on C2 from the committed ncu
+    --set full capture (dram__bytes_read.sum + dram__bytes_write.sum)."""
+    try:
+        d = json.loads((ROOT / "profiles" / "r1b_ncu_full_summary.json").read_text())
+        k = d["spmv_merge_kernel C2 (row-aligned, K=27)"]
+        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
+        rd = float(k["dram__bytes_read.sum"][0]) * scale[k["dram__bytes_read.sum"][1]]
+        wr = float(k["dram__bytes_write.sum"][0]) * scale[k["dram__bytes_write.sum"][1]]
+        if world != 1:
+            return {"traffic": None, "traffic_source": "ncu capture is of the 1-GPU C2 launch"}
+        return {"traffic": rd + wr, "traffic_source": "profiles/r1b_ncu_full_summary.json (ncu --set full, C2 launch)"}
+    except Exception as e:  # noqa: BLE001
+        return {"traffic": None, "traffic_source": f"unavailable: {e}"}
+
+
 def spmv_alg_bytes(m, n, nnz, vsize):
     """4 (col) + s (val) per nonzero, 4 (offset) + s (y) per row,
     s (x) per column read once; plus the final row offset."""
@@ -343,7 +359,7 @@ def msp_arm(args):
             "ops": ops_out,
             "roofline": {"bound": "hbm", "kernel": "spmv_merge_kernel", "achieved": achieved, "peak": peak,
                          "peak_kind": peak_kind, "unit": "GB/s", "frac": achieved / peak,
-                         "alg_bytes_per_launch": by_loc, "traffic": None},
+                         "alg_bytes_per_launch": by_loc, **ncu_traffic(world)},
             "clocks": clocks,
             "gpu_launches": n_launches,
             "e2e": e2e,
