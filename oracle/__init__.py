@@ -26,6 +26,7 @@ _lib = None
 _i32p = np.ctypeslib.ndpointer(np.int32, flags="C_CONTIGUOUS")
 _i64p = np.ctypeslib.ndpointer(np.int64, flags="C_CONTIGUOUS")
 _f64p = np.ctypeslib.ndpointer(np.float64, flags="C_CONTIGUOUS")
+_u64p = np.ctypeslib.ndpointer(np.uint64, flags="C_CONTIGUOUS")
 _vp = ctypes.c_void_p
 
 
@@ -63,6 +64,8 @@ def lib():
                                          _vp, _vp]
         L.oracle_nprods.restype = ctypes.c_int64
         L.oracle_nprods.argtypes = [ctypes.c_int64, _i32p, _i32p]
+        L.oracle_set_op.restype = ctypes.c_int64
+        L.oracle_set_op.argtypes = [ctypes.c_int, _u64p, _vp, ctypes.c_int64, _u64p, _vp, ctypes.c_int64, _vp, _vp]
         L.oracle_row_split.restype = None
         L.oracle_row_split.argtypes = [ctypes.c_int32, _i32p, ctypes.c_int32, _i32p]
         _lib = L
@@ -220,3 +223,33 @@ def check_values(got: np.ndarray, want: np.ndarray, scale: np.ndarray, dtype) ->
         return False, (f"{int(bad.sum())} entries out of tolerance; first at {i}: "
                        f"got {g[ok][i]!r} want {w[ok][i]!r} scale {scale[ok][i]!r}")
     return True, "ok"
+
+
+SET_OPS = {"union": 0, "intersection": 1, "difference": 2, "symmetric_difference": 3}
+
+
+def set_op(op: str, a_keys, b_keys, a_vals=None, b_vals=None):
+    """Multiset operation on sorted keys (key-rank pairs, msp_oracle.c
+    oracle_set_op).  Keys: unsigned 32/64-bit arrays; values: optional arrays
+    of the same length (any 4/8-byte dtype, carried bit-for-bit).
+    Returns (keys, vals or None) in the input dtypes."""
+    kd = np.asarray(a_keys).dtype
+    A = np.ascontiguousarray(np.asarray(a_keys).astype(np.uint64))
+    B = np.ascontiguousarray(np.asarray(b_keys).astype(np.uint64))
+    has_v = a_vals is not None
+    if has_v:
+        vd = np.asarray(a_vals).dtype
+        ut = np.uint32 if vd.itemsize == 4 else np.uint64
+        Av = np.ascontiguousarray(np.asarray(a_vals).view(ut).astype(np.uint64))
+        Bv = np.ascontiguousarray(np.asarray(b_vals).view(ut).astype(np.uint64))
+    L = lib()
+    code = SET_OPS[op]
+    n = L.oracle_set_op(code, A, _ptr(Av) if has_v else None, A.size, B, _ptr(Bv) if has_v else None, B.size,
+                        None, None)
+    C = np.empty(n, dtype=np.uint64)
+    Cv = np.empty(n, dtype=np.uint64) if has_v else None
+    L.oracle_set_op(code, A, _ptr(Av) if has_v else None, A.size, B, _ptr(Bv) if has_v else None, B.size,
+                    _ptr(C), _ptr(Cv) if has_v else None)
+    keys = C.astype(kd)
+    vals = Cv.astype(ut).view(vd) if has_v else None
+    return keys, vals

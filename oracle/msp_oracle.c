@@ -298,3 +298,45 @@ void oracle_row_split(int32_t m, const int32_t *rp, int32_t P, int32_t *starts)
     }
     starts[P] = m;
 }
+
+/* ---------------------------------------------------------------- set ops
+ * Set operations on sorted key lists with duplicates (§8(f) f1):
+ * each key carries a rank inside its run of equal keys, and the i-th copy of
+ * a key in A matches the i-th copy in B ("key-rank pairs").  So for
+ * a key with cA copies in A and cB in B the result holds
+ *   union         max(cA, cB) copies: the min(cA, cB) matched from A, the rest
+ *                 from the longer side;
+ *   intersection  min(cA, cB) copies, from A;
+ *   difference    max(cA - cB, 0) copies: A's copies of rank >= cB;
+ *   sym. diff.    |cA - cB| copies from the longer side,
+ * in ascending key order (the sequential two-pointer walk of Algorithm 1,
+ * A first on ties).  Keys are unsigned 64-bit; values are opaque
+ * 64-bit payloads that travel with their key (A's on a matched pair).
+ * op: 0 union, 1 intersection, 2 difference (A - B), 3 symmetric difference.
+ * C / Cv may be NULL (count only).  Returns the result size. */
+int64_t oracle_set_op(int op, const uint64_t *A, const uint64_t *Av, int64_t nA,
+                      const uint64_t *B, const uint64_t *Bv, int64_t nB, uint64_t *C, uint64_t *Cv)
+{
+    int64_t i = 0, j = 0, n = 0;
+#define EMIT(K, V)                 \
+    do {                           \
+        if (C) C[n] = (K);         \
+        if (Cv) Cv[n] = (V);       \
+        ++n;                       \
+    } while (0)
+    while (i < nA || j < nB) {
+        if (j >= nB || (i < nA && A[i] < B[j])) {           /* A only */
+            if (op == 0 || op == 2 || op == 3) EMIT(A[i], Av ? Av[i] : 0);
+            ++i;
+        } else if (i >= nA || B[j] < A[i]) {                /* B only */
+            if (op == 0 || op == 3) EMIT(B[j], Bv ? Bv[j] : 0);
+            ++j;
+        } else {                                            /* matched pair, same rank */
+            if (op == 0 || op == 1) EMIT(A[i], Av ? Av[i] : 0);
+            ++i;
+            ++j;
+        }
+    }
+#undef EMIT
+    return n;
+}

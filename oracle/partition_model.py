@@ -84,3 +84,36 @@ def row_split(rp: np.ndarray, P: int) -> np.ndarray:
         out.append(int(np.searchsorted(rp, -(-r * nnz // P), side="left")))
     out.append(rp.size - 1)
     return np.array(out, dtype=np.int64)
+
+
+def balanced_path_split_ranked(a, b, d: int) -> tuple[int, int]:
+    """Balanced path for lists WITH duplicate keys (reading R4):
+    items are ordered by (key, rank inside the key's run, A before B), so the
+    i-th copy of a key in `a` is adjacent to the i-th copy in `b` ("keys with
+    matching ranks ... to the same partition").  Returns the split
+    (i, j) of diagonal d; i + j == d + 1 when the cut would separate a matched
+    pair (the starred diagonal takes the B copy).  For unique keys
+    (rank 0 only) this is balanced_path_split (Z23)."""
+    import bisect
+    a = list(a)
+    b = list(b)
+    i, j = merge_path_split(a, b, d)
+    last = [x for x in (a[i - 1] if i > 0 else None, b[j - 1] if j > 0 else None) if x is not None]
+    nxt = [x for x in (a[i] if i < len(a) else None, b[j] if j < len(b) else None) if x is not None]
+    if not last or not nxt or max(last) != min(nxt):
+        return i, j
+    k = max(last)
+    a_lo, a_hi = bisect.bisect_left(a, k), bisect.bisect_right(a, k)
+    b_lo, b_hi = bisect.bisect_left(b, k), bisect.bisect_right(b, k)
+    ca, cb = a_hi - a_lo, b_hi - b_lo
+    p = (i - a_lo) + (j - b_lo)          # items of key k before the cut
+    m = min(ca, cb)
+    if p <= 2 * m:
+        ia, ib = (p + 1) // 2, p // 2
+        if ia > ib:                      # cut between (k, r) in A and (k, r) in B
+            ib += 1
+    elif ca > cb:
+        ia, ib = p - cb, cb
+    else:
+        ia, ib = ca, p - ca
+    return a_lo + ia, b_lo + ib
