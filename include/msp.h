@@ -189,6 +189,38 @@ msp_status msp_csr_check(const msp_csr *A, int require_sorted_unique, int32_t *f
                          void *ws, size_t ws_bytes, void *stream);
 
 /* ------------------------------------------------------------------------
+ * Set operations on sorted key lists (the paper's second
+ * contribution, Fig 2).  A_keys[nA], B_keys[nB]: device,
+ * sorted ascending as unsigned integers of key_bytes (4 or 8) bytes;
+ * duplicates allowed.  A_vals / B_vals: device payloads of val_bytes (0, 4 or
+ * 8; NULL when 0) per key, carried bit-for-bit.  Duplicates are key-rank
+ * pairs: the r-th copy of a key in A matches the r-th copy in B (P:700-712,
+ * reading R4), so with cA / cB copies of a key the result holds
+ *   MSP_SET_UNION                 max(cA, cB) copies (matched from A),
+ *   MSP_SET_INTERSECTION          min(cA, cB) copies (from A),
+ *   MSP_SET_DIFFERENCE            max(cA - cB, 0) copies (A - B),
+ *   MSP_SET_SYMMETRIC_DIFFERENCE  |cA - cB| copies (longer side),
+ * ascending.  C_keys / C_vals: device, capacity C_capacity entries, which
+ * must be at least nA + nB (union, symmetric difference), min(nA, nB)
+ * (intersection) or nA (difference), else MSP_ERR_SHAPE.  *nC_host receives
+ * the result size.  ws: msp_set_op_workspace() bytes, caller-owned.
+ * Synchronises the stream (returns the size).  Unsorted input gives an
+ * unspecified (but memory-safe) result.
+ * ------------------------------------------------------------------------ */
+typedef enum {
+    MSP_SET_UNION = 0,
+    MSP_SET_INTERSECTION = 1,
+    MSP_SET_DIFFERENCE = 2,
+    MSP_SET_SYMMETRIC_DIFFERENCE = 3
+} msp_set_op;
+
+msp_status msp_set_op_workspace(int64_t nA, int64_t nB, size_t *bytes);
+msp_status msp_set_operation(msp_set_op op, const void *A_keys, const void *A_vals, int64_t nA,
+                             const void *B_keys, const void *B_vals, int64_t nB, int32_t key_bytes,
+                             int32_t val_bytes, void *C_keys, void *C_vals, int64_t C_capacity,
+                             int64_t *nC_host, void *ws, size_t ws_bytes, void *stream);
+
+/* ------------------------------------------------------------------------
  * Multi-GPU helpers.  Row blocks are balanced by nnz:
  * rank r owns rows [R_r, R_{r+1}), R_r = lower_bound(row_offsets,
  * ceil(r * nnz / P)), R_0 = 0, R_P = nrows.  row_offsets_host is a HOST

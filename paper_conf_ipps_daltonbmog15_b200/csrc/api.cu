@@ -297,4 +297,49 @@ msp_status msp_rebase_offsets(const int32_t *in, int32_t *out, int64_t n, int64_
     return rebase_run(in, out, n, base, as_stream(stream));
 }
 
+msp_status msp_set_op_workspace(int64_t nA, int64_t nB, size_t *bytes)
+{
+    clear_error();
+    if (!bytes || nA < 0 || nB < 0) return MSP_ERR_ARG;
+    *bytes = set_op_ws_bytes(nA, nB);
+    return MSP_OK;
+}
+
+msp_status msp_set_operation(msp_set_op op, const void *A_keys, const void *A_vals, int64_t nA, const void *B_keys,
+                             const void *B_vals, int64_t nB, int32_t key_bytes, int32_t val_bytes, void *C_keys,
+                             void *C_vals, int64_t C_capacity, int64_t *nC_host, void *ws, size_t ws_bytes,
+                             void *stream)
+{
+    clear_error();
+    if (!nC_host || nA < 0 || nB < 0 || int(op) < 0 || int(op) > 3) return MSP_ERR_ARG;
+    if (key_bytes != 4 && key_bytes != 8) {
+        set_error("set op: key_bytes must be 4 or 8");
+        return MSP_ERR_DTYPE;
+    }
+    if (val_bytes != 0 && val_bytes != 4 && val_bytes != 8) {
+        set_error("set op: val_bytes must be 0, 4 or 8");
+        return MSP_ERR_DTYPE;
+    }
+    if ((nA > 0 && !A_keys) || (nB > 0 && !B_keys) || (val_bytes && ((nA > 0 && !A_vals) || (nB > 0 && !B_vals)))) {
+        set_error("set op: NULL input");
+        return MSP_ERR_ARG;
+    }
+    if (nA + nB > (int64_t(1) << 40)) {
+        set_error("set op: inputs too large");
+        return MSP_ERR_OVERFLOW;
+    }
+    const int64_t bound = op == MSP_SET_INTERSECTION ? (nA < nB ? nA : nB) : op == MSP_SET_DIFFERENCE ? nA : nA + nB;
+    if (C_capacity < bound) {
+        set_error("set op: C capacity %lld below the result bound %lld", (long long)C_capacity, (long long)bound);
+        return MSP_ERR_SHAPE;
+    }
+    if (bound > 0 && (!C_keys || (val_bytes && !C_vals))) {
+        set_error("set op: NULL output");
+        return MSP_ERR_ARG;
+    }
+    if (!ws && nA + nB > 0) return MSP_ERR_ARG;
+    return set_op_run(int(op), A_keys, A_vals, nA, B_keys, B_vals, nB, key_bytes, val_bytes, C_keys, C_vals, nC_host,
+                      ws, ws_bytes, as_stream(stream));
+}
+
 }  // extern "C"

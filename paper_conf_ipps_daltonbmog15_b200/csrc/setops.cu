@@ -1,0 +1,324 @@
+// setops.cu -- balanced-path set operations on sorted key lists (sm_100a).
+//
+// Paper: Section III-B, the paper's second contribution
+// and its Fig 2 benchmark: union, intersection, difference and symmetric
+// difference of two sorted lists with duplicates, keys only or key-value
+// pairs, 32- or 64-bit.  Duplicates are key-rank pairs: the r-th copy of a key
+// in A matches the r-th copy in B, so items are ordered by
+// (key, rank, A first) and balanced path keeps every matched pair on one side
+// of every cut -- reading R4; for unique keys it is the Z23 shift.
+//
+// B200 design: ONE pass over the data.
+//   * partition kernel: one thread per tile boundary, merge-path search over
+//     A and B in global memory, then the balanced-path fix-up inside the run
+//     of equal keys the cut falls in;
+//   * tile kernel (one CTA per tile of T items, tiles claimed in order by an
+//     atomic ticket): coalesced staging of the tile's A and B windows (keys
+//     and values) in shared memory, per-thread balanced-path split in shared
+//     memory, serial walk counting the outputs, CTA scan, decoupled look-back
+//     over the tiles for the global output offset, second walk writing the
+//     outputs.  The result size comes back with the last tile's prefix.
+#include <algorithm>
+#include <climits>
+#include <cstdint>
+
+#include "common.cuh"
+#include "internal.h"
+
+namespace msp {
+namespace {
+
+constexpr int SET_NT = 256;
+constexpr int SET_IPT = 12;
+constexpr int SET_T = SET_NT * SET_IPT;  // merge items per tile (+1 for a starred cut)
+
+struct Cut {
+    int64_t i, j;
+};
+
+// Balanced-path cut of diagonal d over key arrays A[0..na), B[0..nb)
+// (global or shared memory, any key type).  See partition_model.py
+// balanced_path_split_ranked for the reference statement of the rule.
+template <typename KT, class LA, class LB>
+__device__ __forceinline__ Cut balanced_cut(LA A, int64_t na, LB B, int64_t nb, int64_t d)
+{
+    int64_t lo = d > nb ? d - nb : 0, hi = d < na ? d : na;
+    while (lo < hi) {  // merge path, A first on ties (Alg. 1)
+        const int64_t mid = (lo + hi) >> 1;
+        if (A(mid) <= B(d - mid - 1)) lo = mid + 1;
+        else hi = mid;
+    }
+    int64_t i = lo, j = d - lo;
+    const bool hl = i > 0 || j > 0, hn = i < na || j < nb;
+    if (!hl || !hn) return Cut{i, j};
+    KT last = 0, next = ~KT(0);
+    if (i > 0) last = A(i - 1);
+    if (j > 0 && B(j - 1) > last) last = B(j - 1);
+    if (i < na) next = A(i);
+    if (j < nb && B(j) < next) next = B(j);
+    if (last != next) return Cut{i, j};  // the cut is between two keys
+    const KT k = last;
+    auto lower = [&](auto X, int64_t l, int64_t h) {  // first index in [l, h) with X >= k
+        while (l < h) {
+            const int64_t m = (l + h) >> 1;
+            if (X(m) < k) l = m + 1;
+            else h = m;
+        }
+        return l;
+    };
+    auto upper = [&](auto X, int64_t l, int64_t h) {  // first index in [l, h) with X > k
+        while (l < h) {
+            const int64_t m = (l + h) >> 1;
+            if (X(m) <= k) l = m + 1;
+            else h = m;
+        }
+        return l;
+    };
+    const int64_t a_lo = lower(A, 0, i), a_hi = upper(A, i, na);
+    const int64_t b_lo = lower(B, 0, j), b_hi = upper(B, j, nb);
+    const int64_t ca = a_hi - a_lo, cb = b_hi - b_lo;
+    const int64_t p = (i - a_lo) + (j - b_lo);  // items of key k before the cut
+    const int64_t mm = ca < cb ? ca : cb;
+    int64_t ia, ib;
+    if (p <= 2 * mm) {
+        ia = (p + 1) >> 1;
+        ib = p >> 1;
+        if (ia > ib) ++ib;  // starred: the matched B copy joins the left side
+    } else if (ca > cb) {
+        ia = p - cb;
+        ib = cb;
+    } else {
+        ia = ca;
+        ib = p - ca;
+    }
+    return Cut{a_lo + ia, b_lo + ib};
+}
+
+template <typename KT>
+__global__ void set_partition_kernel(const KT *__restrict__ A, int64_t na, const KT *__restrict__ B, int64_t nb,
+                                     int64_t ntiles, Cut *__restrict__ cuts)
+{
+    const int64_t total = na + nb;
+    for (int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; k <= ntiles;
+         k += int64_t(gridDim.x) * blockDim.x) {
+        const int64_t d = k * SET_T < total ? k * SET_T : total;
+        cuts[k] = balanced_cut<KT>([&](int64_t x) { return A[x]; }, na, [&](int64_t x) { return B[x]; }, nb, d);
+    }
+}
+
+template <int VB> struct ValT { using T = uint32_t; };
+template <> struct ValT<8> { using T = uint64_t; };
+
+template <typename KT, int VB>
+struct SetSmem {
+    KT ka[SET_T + 2];
+    KT kb[SET_T + 2];
+    typename ValT<VB>::T va[VB ? SET_T + 2 : 1];
+    typename ValT<VB>::T vb[VB ? SET_T + 2 : 1];
+    int cut_i[SET_NT + 1], cut_j[SET_NT + 1];
+    int wsum[SET_NT / 32];
+    int64_t base;
+    int tile;
+};
+
+constexpr uint64_t ST_AGG = 1ull << 62, ST_PRE = 2ull << 62, ST_VAL = (1ull << 62) - 1;
+
+// op: 0 union, 1 intersection, 2 difference (A - B), 3 symmetric difference
+template <typename KT, int VB, int OP>
+__global__ void __launch_bounds__(SET_NT)
+set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t na, const KT *__restrict__ B,
+                const void *__restrict__ Bv, int64_t nb, const Cut *__restrict__ cuts, int64_t ntiles,
+                uint64_t *__restrict__ states, unsigned *__restrict__ ticket, KT *__restrict__ C,
+                void *__restrict__ Cv, int64_t *__restrict__ nC)
+{
+    using VT = typename ValT<VB>::T;
+    constexpr bool EA = (OP == 0 || OP == 2 || OP == 3), EB = (OP == 0 || OP == 3), EM = (OP == 0 || OP == 1);
+    extern __shared__ __align__(16) char smem_raw[];
+    SetSmem<KT, VB> &S = *reinterpret_cast<SetSmem<KT, VB> *>(smem_raw);
+    const int tid = threadIdx.x;
+    if (tid == 0) S.tile = int(atomicAdd(ticket, 1u));  // tiles in claim order: look-back never waits on an unstarted tile
+    __syncthreads();
+    const int tile = S.tile;
+    const Cut c0 = cuts[tile], c1 = cuts[tile + 1];
+    const int la = int(c1.i - c0.i), lb = int(c1.j - c0.j);
+    for (int x = tid; x < la; x += SET_NT) {
+        S.ka[x] = A[c0.i + x];
+        if constexpr (VB > 0) S.va[x] = static_cast<const VT *>(Av)[c0.i + x];
+    }
+    for (int x = tid; x < lb; x += SET_NT) {
+        S.kb[x] = B[c0.j + x];
+        if constexpr (VB > 0) S.vb[x] = static_cast<const VT *>(Bv)[c0.j + x];
+    }
+    __syncthreads();
+    {  // this thread's cut inside the tile (windows clipped to the tile: consistent, R4)
+        const int d = min(tid * SET_IPT, la + lb);
+        const Cut c = balanced_cut<KT>([&](int64_t x) { return S.ka[x]; }, la, [&](int64_t x) { return S.kb[x]; },
+                                       lb, d);
+        S.cut_i[tid] = int(c.i);
+        S.cut_j[tid] = int(c.j);
+        if (tid == 0) {
+            S.cut_i[SET_NT] = la;
+            S.cut_j[SET_NT] = lb;
+        }
+    }
+    __syncthreads();
+    // a starred cut may pass the next thread's nominal diagonal: clamp (monotone)
+    int ia0 = S.cut_i[tid], ib0 = S.cut_j[tid];
+    int ia1 = max(S.cut_i[tid + 1], ia0), ib1 = max(S.cut_j[tid + 1], ib0);
+    auto walk = [&](auto &&emit) {
+        int ia = ia0, ib = ib0;
+        while (ia < ia1 || ib < ib1) {
+            const bool ra = ia < ia1, rb = ib < ib1;
+            if (ra && (!rb || S.ka[ia] < S.kb[ib])) {
+                if (EA) emit(true, ia);
+                ++ia;
+            } else if (rb && (!ra || S.kb[ib] < S.ka[ia])) {
+                if (EB) emit(false, ib);
+                ++ib;
+            } else {  // matched key-rank pair: A's copy
+                if (EM) emit(true, ia);
+                ++ia;
+                ++ib;
+            }
+        }
+    };
+    int cnt = 0;
+    walk([&](bool, int) { ++cnt; });
+    int tot;
+    const int off = block_exclusive_sum<int, SET_NT / 32>(cnt, S.wsum, 1, &tot);
+    if (tid == 0) {  // decoupled look-back over the tiles
+        int64_t excl = 0;
+        if (tile == 0) {
+            __threadfence();
+            atomicExch(reinterpret_cast<unsigned long long *>(&states[0]), (unsigned long long)(ST_PRE | uint64_t(tot)));
+        } else {
+            atomicExch(reinterpret_cast<unsigned long long *>(&states[tile]), (unsigned long long)(ST_AGG | uint64_t(tot)));
+            for (int k = tile - 1; k >= 0;) {
+                const uint64_t st = *reinterpret_cast<volatile uint64_t *>(&states[k]);
+                if ((st & ~ST_VAL) == 0) continue;  // predecessor not published yet
+                excl += int64_t(st & ST_VAL);
+                if (st & ST_PRE) break;
+                --k;
+            }
+            __threadfence();
+            atomicExch(reinterpret_cast<unsigned long long *>(&states[tile]),
+                       (unsigned long long)(ST_PRE | uint64_t(excl + tot)));
+        }
+        S.base = excl;
+        if (tile == ntiles - 1) *nC = excl + tot;
+    }
+    __syncthreads();
+    int64_t pos = S.base + off;
+    walk([&](bool fromA, int x) {
+        C[pos] = fromA ? S.ka[x] : S.kb[x];
+        if constexpr (VB > 0) static_cast<VT *>(Cv)[pos] = fromA ? S.va[x] : S.vb[x];
+        ++pos;
+    });
+}
+
+struct SetWs {
+    Cut *cuts;
+    uint64_t *states;
+    unsigned *ticket;
+    int64_t *nC;
+    int64_t ntiles;
+    size_t bytes;
+};
+
+SetWs carve(int64_t na, int64_t nb, void *ws, size_t bytes, bool *ok)
+{
+    SetWs w;
+    const int64_t items = na + nb;
+    w.ntiles = items > 0 ? ceil_div(items, SET_T) : 0;
+    Carve cv(ws, bytes);
+    w.ticket = cv.take<unsigned>(4);
+    w.nC = cv.take<int64_t>(1);
+    w.states = cv.take<uint64_t>(size_t(w.ntiles > 0 ? w.ntiles : 1));
+    w.cuts = cv.take<Cut>(size_t(w.ntiles + 1));
+    w.bytes = cv.off;
+    *ok = cv.ok();
+    return w;
+}
+
+template <typename KT, int VB, int OP>
+msp_status launch_tiles(const void *A, const void *Av, int64_t na, const void *B, const void *Bv, int64_t nb,
+                        const SetWs &w, void *C, void *Cv, cudaStream_t s)
+{
+    auto kern = set_tile_kernel<KT, VB, OP>;
+    const int smem = int(sizeof(SetSmem<KT, VB>));
+    static int configured = 0;
+    if (!configured) {
+        msp_status st = cuda_check(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem),
+                                   "set op: smem");
+        if (st != MSP_OK) return st;
+        configured = 1;
+    }
+    kern<<<unsigned(w.ntiles), SET_NT, smem, s>>>(static_cast<const KT *>(A), Av, na, static_cast<const KT *>(B), Bv,
+                                                  nb, w.cuts, w.ntiles, w.states, w.ticket, static_cast<KT *>(C), Cv,
+                                                  w.nC);
+    return last_launch("set_tile_kernel");
+}
+
+template <typename KT, int VB>
+msp_status launch_op(int op, const void *A, const void *Av, int64_t na, const void *B, const void *Bv, int64_t nb,
+                     const SetWs &w, void *C, void *Cv, cudaStream_t s)
+{
+    switch (op) {
+    case 0: return launch_tiles<KT, VB, 0>(A, Av, na, B, Bv, nb, w, C, Cv, s);
+    case 1: return launch_tiles<KT, VB, 1>(A, Av, na, B, Bv, nb, w, C, Cv, s);
+    case 2: return launch_tiles<KT, VB, 2>(A, Av, na, B, Bv, nb, w, C, Cv, s);
+    default: return launch_tiles<KT, VB, 3>(A, Av, na, B, Bv, nb, w, C, Cv, s);
+    }
+}
+
+template <typename KT>
+msp_status launch_kv(int op, int vb, const void *A, const void *Av, int64_t na, const void *B, const void *Bv,
+                     int64_t nb, const SetWs &w, void *C, void *Cv, cudaStream_t s)
+{
+    if (vb == 0) return launch_op<KT, 0>(op, A, Av, na, B, Bv, nb, w, C, Cv, s);
+    if (vb == 4) return launch_op<KT, 4>(op, A, Av, na, B, Bv, nb, w, C, Cv, s);
+    return launch_op<KT, 8>(op, A, Av, na, B, Bv, nb, w, C, Cv, s);
+}
+
+}  // namespace
+
+size_t set_op_ws_bytes(int64_t na, int64_t nb)
+{
+    bool ok;
+    return carve(na, nb, nullptr, SIZE_MAX, &ok).bytes + 256;
+}
+
+msp_status set_op_run(int op, const void *A, const void *Av, int64_t na, const void *B, const void *Bv, int64_t nb,
+                      int key_bytes, int val_bytes, void *C, void *Cv, int64_t *nC_host, void *ws, size_t ws_bytes,
+                      cudaStream_t s)
+{
+    bool ok;
+    SetWs w = carve(na, nb, ws, ws_bytes, &ok);
+    if (!ok) return MSP_ERR_WORKSPACE;
+    if (w.ntiles == 0) {
+        *nC_host = 0;
+        return MSP_OK;
+    }
+    msp_status st = cuda_check(cudaMemsetAsync(ws, 0, reinterpret_cast<char *>(w.cuts) - static_cast<char *>(ws), s),
+                               "set op: clear look-back state");
+    if (st != MSP_OK) return st;
+    {
+        const unsigned blocks = unsigned(std::min<int64_t>(ceil_div(w.ntiles + 1, 256), 148 * 8));
+        if (key_bytes == 4)
+            set_partition_kernel<uint32_t><<<blocks, 256, 0, s>>>(static_cast<const uint32_t *>(A), na,
+                                                                  static_cast<const uint32_t *>(B), nb, w.ntiles, w.cuts);
+        else
+            set_partition_kernel<uint64_t><<<blocks, 256, 0, s>>>(static_cast<const uint64_t *>(A), na,
+                                                                  static_cast<const uint64_t *>(B), nb, w.ntiles, w.cuts);
+        st = last_launch("set_partition_kernel");
+        if (st != MSP_OK) return st;
+    }
+    st = (key_bytes == 4) ? launch_kv<uint32_t>(op, val_bytes, A, Av, na, B, Bv, nb, w, C, Cv, s)
+                          : launch_kv<uint64_t>(op, val_bytes, A, Av, na, B, Bv, nb, w, C, Cv, s);
+    if (st != MSP_OK) return st;
+    st = cuda_check(cudaMemcpyAsync(nC_host, w.nC, sizeof(int64_t), cudaMemcpyDeviceToHost, s), "set op: size");
+    if (st != MSP_OK) return st;
+    return cuda_check(cudaStreamSynchronize(s), "set op: sync");
+}
+
+}  // namespace msp

@@ -246,3 +246,45 @@ def rebase_offsets(rp: torch.Tensor, base: int, out: torch.Tensor | None = None)
     check("msp_rebase_offsets", lib().msp_rebase_offsets(rp.data_ptr(), out.data_ptr(), rp.numel(), int(base),
                                                          _stream_ptr(rp.device)))
     return out
+
+
+# ----------------------------------------------------------------- set operations
+
+SET_OPS = {"union": 0, "intersection": 1, "difference": 2, "symmetric_difference": 3}
+_KEY_T = {torch.int32: 4, torch.int64: 8, torch.uint32: 4, torch.uint64: 8}
+
+
+def set_operation(op: str, a_keys: torch.Tensor, b_keys: torch.Tensor, a_vals: torch.Tensor | None = None,
+                  b_vals: torch.Tensor | None = None, stream=None):
+    """Balanced-path set operation on sorted key lists: keys are
+    compared as unsigned 32/64-bit integers (int32/int64 tensors are
+    reinterpreted), duplicates are key-rank pairs.  Returns (keys, vals or
+    None), trimmed to the result size (msp_set_operation synchronises)."""
+    code = SET_OPS[op]
+    if a_keys.dtype != b_keys.dtype or a_keys.dtype not in _KEY_T:
+        raise ValueError("keys must share a 32/64-bit integer dtype")
+    if not (a_keys.is_contiguous() and b_keys.is_contiguous()) or a_keys.device != b_keys.device:
+        raise ValueError("keys must be contiguous tensors on one device")
+    kb = _KEY_T[a_keys.dtype]
+    vb = 0
+    if a_vals is not None:
+        if b_vals is None or a_vals.dtype != b_vals.dtype or a_vals.element_size() not in (4, 8):
+            raise ValueError("values: both sides, one 4/8-byte dtype")
+        if a_vals.numel() != a_keys.numel() or b_vals.numel() != b_keys.numel():
+            raise ValueError("one value per key")
+        vb = a_vals.element_size()
+    na, nb = a_keys.numel(), b_keys.numel()
+    bound = min(na, nb) if op == "intersection" else na if op == "difference" else na + nb
+    dev = a_keys.device
+    ck = torch.empty(max(bound, 1), dtype=a_keys.dtype, device=dev)
+    cv = torch.empty(max(bound, 1), dtype=a_vals.dtype, device=dev) if vb else None
+    n = ctypes.c_size_t(0)
+    check("msp_set_op_workspace", lib().msp_set_op_workspace(na, nb, ctypes.byref(n)))
+    ws = workspace(int(n.value), dev, "setop", stream)
+    nc = ctypes.c_int64(0)
+    check("msp_set_operation", lib().msp_set_operation(
+        code, a_keys.data_ptr(), a_vals.data_ptr() if vb else None, na, b_keys.data_ptr(),
+        b_vals.data_ptr() if vb else None, nb, kb, vb, ck.data_ptr(), cv.data_ptr() if vb else None, bound,
+        ctypes.byref(nc), ws.data_ptr(), ws.numel(), _stream_ptr(dev, stream)))
+    k = int(nc.value)
+    return ck[:k], (cv[:k] if vb else None)
