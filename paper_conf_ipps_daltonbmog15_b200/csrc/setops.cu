@@ -29,7 +29,10 @@ namespace msp {
 namespace {
 
 constexpr int SET_NT = 256;
-constexpr int SET_IPT = 12;
+#ifndef MSP_SET_IPT
+#define MSP_SET_IPT 12
+#endif
+constexpr int SET_IPT = MSP_SET_IPT;
 constexpr int SET_T = SET_NT * SET_IPT;  // merge items per tile (+1 for a starred cut)
 
 struct Cut {

@@ -104,3 +104,18 @@ def test_capacity_and_dtype_errors():
                                  ctypes.byref(nc), ws.data_ptr(), ws.numel(), None)
     assert st == 2  # MSP_ERR_DTYPE
     assert MspError
+
+
+@pytest.mark.parametrize("kind", ["keys-32", "pairs-64"])
+def test_fig2_scale(kind):
+    """The Fig 2 workload shape at 2e7 inputs (union, inputs split evenly,
+    uniform keys below 2^30 as tools/setops_bench.py draws them), exact."""
+    rng = np.random.default_rng(2)
+    kd = np.uint32 if kind == "keys-32" else np.uint64
+    n = 10**7
+    a = np.sort(rng.integers(0, 2**30, size=n)).astype(kd)
+    b = np.sort(rng.integers(0, 2**30, size=n)).astype(kd)
+    if kind == "pairs-64":
+        check("union", a, b, np.arange(n, dtype=np.int64), -np.arange(n, dtype=np.int64), label="2e7 pairs-64")
+    else:
+        check("union", a, b, label="2e7 keys-32")
