@@ -33,6 +33,8 @@ ROOT = Path(__file__).resolve().parent
 sys.path.insert(0, str(ROOT))
 
 HBM_FALLBACK = 6650.0
+METRIC = "SpMV GB/s (algorithmic bytes / time) on C2; SpAdd input nnz/s, SpGEMM products/s beside"
+WORKLOAD_C2 = "C2: 3D Poisson 27-point 100^3 fp64 (BJ:8)"
 
 
 def peaks():
@@ -157,11 +159,11 @@ def reference_arm(args):
     if rank != 0:
         return 0
     res = cpu_baseline(budget_s=max(2.0, 6.0 * (args.steps + args.warmup) / 20))
-    line = {"impl": "reference", "metric": "SpMV GB/s (algorithmic bytes / time)", "value": res["value"],
+    line = {"impl": "reference", "metric": METRIC, "value": res["value"],
             "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-            "data": "synthetic", "config": {"workload": "C2: 3D Poisson 27-point 100^3 fp64",
-                                            "kernel": "CPU oracle (scalar CSR, P:364-370)"},
+            "data": "synthetic (seeded generators, gen/)",
+            "config": {"workload": WORKLOAD_C2, "kernel": "CPU oracle (scalar CSR, P:364-370), host cores"},
             "cpu_baseline": res, "e2e": {"value": res["value"], "unit": "GB/s", "h2d_bytes_per_step": 0,
                                           "d2h_bytes_per_step": 0}}
     print(json.dumps(line))
@@ -352,11 +354,11 @@ def msp_arm(args):
         cpu = cpu_baseline(budget_s=10.0)
     if rank == 0:
         line = {
-            "metric": "SpMV GB/s (algorithmic bytes / time) on C2; SpAdd input nnz/s, SpGEMM products/s beside",
+            "metric": METRIC,
             "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": step_ms, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "f64", "data": "synthetic (seeded generators, gen/)",
-            "config": {"workload": "C2: 3D Poisson 27-point 100^3 fp64 (BJ:8)" if world == 1 else
+            "config": {"workload": WORKLOAD_C2 if world == 1 else
                        f"3D Poisson 27-point 100x100x{100 * world} fp64, 100^3 rows per rank",
                        "ops": ",".join(k for k in ("spmv", "spadd", "spgemm") if k == "spmv" or have[k]),
                        "spmv_reps_per_step": args.spmv_reps, "parallelism": f"row blocks x{world}",
