@@ -63,6 +63,7 @@ struct CtaRecord {  // one per CTA in the workspace
 template <typename V, int NW_, int STAGES_, int RSLOTS_, int MINB_>
 struct Cfg {
     static constexpr bool ROWK = false;
+    static constexpr bool PREFETCH = false;  // L2 prefetch measured 4 % slower on C3 for this walk
     static constexpr int NW = NW_;
     static constexpr int K = 8;
     static constexpr int WSPAN = 32 * K;                 // products per worker warp
@@ -93,6 +94,7 @@ struct Cfg {
 template <typename V, int NW_, int K_, int STAGES_, int MINB_>
 struct CfgK {
     static constexpr bool ROWK = true;
+    static constexpr bool PREFETCH = true;
     static constexpr int NW = NW_;
     static constexpr int K = K_;
     static constexpr int WSPAN = 32 * K;
@@ -274,7 +276,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
         int j_s = int(d_begin - i_s);
         int prev_rows = 0;
         const int64_t j_cta_end = min64(nnz, d_end);  // upper bound for prefetching
-        if (lane == 0) {                               // warm the first two tiles' data in L2
+        if (C::PREFETCH && lane == 0) {                // warm the first two tiles' data in L2
             prefetch_range<4>(rp, i_s, min64(int64_t(m) + 1, int64_t(i_s) + 2 * C::T + 1));
             prefetch_range<4>(col, j_s, min64(j_cta_end, int64_t(j_s) + 2 * C::T));
             prefetch_range<int(sizeof(V))>(val, j_s, min64(j_cta_end, int64_t(j_s) + 2 * C::T));
@@ -287,7 +289,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             const int i_e = warp_grid_search_guess(rp, de, lo, hi, i_s + prev_rows, lane);
             const int j_e = int(de - i_e);
             prev_rows = i_e - i_s;
-            if (lane == 0) {  // keep the data two tiles ahead streaming into L2
+            if (C::PREFETCH && lane == 0) {  // keep the data two tiles ahead streaming into L2
                 const int64_t rr = max(prev_rows, 32);
                 prefetch_range<4>(rp, int64_t(i_e) + rr, min64(int64_t(m) + 1, int64_t(i_e) + 3 * rr + 1));
                 prefetch_range<4>(col, int64_t(j_e) + C::T, min64(j_cta_end, int64_t(j_e) + 2 * C::T));
