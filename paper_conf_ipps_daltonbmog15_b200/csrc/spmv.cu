@@ -63,7 +63,6 @@ struct CtaRecord {  // one per CTA in the workspace
 template <typename V, int NW_, int STAGES_, int RSLOTS_, int MINB_>
 struct Cfg {
     static constexpr bool ROWK = false;
-    static constexpr bool PREFETCH = false;  // L2 prefetch measured 4 % slower on C3 for this walk
     static constexpr int NW = NW_;
     static constexpr int K = 8;
     static constexpr int WSPAN = 32 * K;                 // products per worker warp
@@ -94,7 +93,6 @@ struct Cfg {
 template <typename V, int NW_, int K_, int STAGES_, int MINB_>
 struct CfgK {
     static constexpr bool ROWK = true;
-    static constexpr bool PREFETCH = true;
     static constexpr int NW = NW_;
     static constexpr int K = K_;
     static constexpr int WSPAN = 32 * K;
@@ -166,21 +164,6 @@ __device__ __forceinline__ void mbar_wait_backoff(uint64_t *bar, uint32_t parity
 {
     while (!mbar_try_wait(bar, parity)) {
     }
-}
-
-__device__ __forceinline__ void prefetch_l2(const void *p, uint32_t bytes)
-{
-    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
-}
-
-// L2 prefetch of elements [lo, hi) of an array (16-byte aligned interior).
-template <int ES>
-__device__ __forceinline__ void prefetch_range(const void *base, int64_t lo, int64_t hi)
-{
-    if (hi <= lo) return;
-    const uintptr_t s = (reinterpret_cast<uintptr_t>(base) + uintptr_t(lo) * ES + 15) & ~uintptr_t(15);
-    const uintptr_t e = (reinterpret_cast<uintptr_t>(base) + uintptr_t(hi) * ES) & ~uintptr_t(15);
-    if (e > s) prefetch_l2(reinterpret_cast<const void *>(s), uint32_t(e - s));
 }
 
 // Split search with a guess: probe the 32 consecutive rows around `g` first
@@ -275,12 +258,6 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
         int i_s = warp_grid_search(rp, d_begin, int(max64(0, d_begin - nnz)), int(min64(d_begin, m)), lane);
         int j_s = int(d_begin - i_s);
         int prev_rows = 0;
-        const int64_t j_cta_end = min64(nnz, d_end);  // upper bound for prefetching
-        if (C::PREFETCH && lane == 0) {                // warm the first two tiles' data in L2
-            prefetch_range<4>(rp, i_s, min64(int64_t(m) + 1, int64_t(i_s) + 2 * C::T + 1));
-            prefetch_range<4>(col, j_s, min64(j_cta_end, int64_t(j_s) + 2 * C::T));
-            prefetch_range<int(sizeof(V))>(val, j_s, min64(j_cta_end, int64_t(j_s) + 2 * C::T));
-        }
         for (int t = 0; t < ntiles; ++t) {
             const int stage = t % C::STAGES;
             const int64_t de = min64(d_begin + int64_t(t + 1) * C::T, d_end);
@@ -289,12 +266,6 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             const int i_e = warp_grid_search_guess(rp, de, lo, hi, i_s + prev_rows, lane);
             const int j_e = int(de - i_e);
             prev_rows = i_e - i_s;
-            if (C::PREFETCH && lane == 0) {  // keep the data two tiles ahead streaming into L2
-                const int64_t rr = max(prev_rows, 32);
-                prefetch_range<4>(rp, int64_t(i_e) + rr, min64(int64_t(m) + 1, int64_t(i_e) + 3 * rr + 1));
-                prefetch_range<4>(col, int64_t(j_e) + C::T, min64(j_cta_end, int64_t(j_e) + 2 * C::T));
-                prefetch_range<int(sizeof(V))>(val, int64_t(j_e) + C::T, min64(j_cta_end, int64_t(j_e) + 2 * C::T));
-            }
             if (t >= C::STAGES) mbar_wait_backoff(&empty[stage], ((t / C::STAGES) - 1) & 1);
             char *sb = stages + size_t(stage) * C::STAGE_BYTES;
             const int wr_end = min(i_e + 1, m);
