@@ -562,14 +562,16 @@ long_chunk_kernel(const int32_t *__restrict__ Arp, const int32_t *__restrict__ A
 }
 
 // One merge pass: runs of `w` entries inside each long row are merged
-// pairwise (stable, left run first).  Each thread produces 16 outputs.
+// pairwise (stable, left run first).  Outputs [e, e_end) by one thread: a
+// merge-path search in global memory, then a serial merge (the fallback for
+// CTAs whose output range crosses a pair or a row boundary).
 template <bool NUM>
-__global__ void long_merge_kernel(int64_t LP, int64_t nlong, const int64_t *__restrict__ longO,
-                                  const int64_t *__restrict__ longP, int64_t w, const int32_t *__restrict__ Xc,
-                                  const double *__restrict__ Xv, int32_t *__restrict__ Yc, double *__restrict__ Yv)
+__device__ __forceinline__ void long_merge_thread(int64_t e, int64_t e_end, int64_t nlong,
+                                                  const int64_t *__restrict__ longO, const int64_t *__restrict__ longP,
+                                                  int64_t w, const int32_t *__restrict__ Xc,
+                                                  const double *__restrict__ Xv, int32_t *__restrict__ Yc,
+                                                  double *__restrict__ Yv)
 {
-    int64_t e = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) * 16;
-    const int64_t e_end = dmin(e + 16, LP);
     while (e < e_end) {
         int64_t lo = 0, hi = nlong;
         while (hi - lo > 1) {
@@ -605,6 +607,91 @@ __global__ void long_merge_kernel(int64_t LP, int64_t nlong, const int64_t *__re
             }
         }
         e += n;
+    }
+}
+
+// CTA-level merge pass (P:1154-1170 global merge of the sorted runs): each CTA
+// owns LM_T consecutive outputs.  When they lie inside one pair of runs (the
+// common case: pairs are >= 2 * GM_TL = 16K long), two merge-path searches
+// bound the CTA's windows of both runs, the windows are staged in shared
+// memory with coalesced loads, and every thread merges 16 outputs from shared
+// memory; other CTAs fall back to the per-thread merge.
+constexpr int LM_NT = 256, LM_IPT = 12, LM_T = LM_NT * LM_IPT;  // 36 KB of static shared memory
+
+template <bool NUM>
+__global__ void __launch_bounds__(LM_NT)
+long_merge_kernel(int64_t LP, int64_t nlong, const int64_t *__restrict__ longO, const int64_t *__restrict__ longP,
+                  int64_t w, const int32_t *__restrict__ Xc, const double *__restrict__ Xv, int32_t *__restrict__ Yc,
+                  double *__restrict__ Yv)
+{
+    __shared__ int32_t sc[LM_T];
+    __shared__ double sv[NUM ? LM_T : 1];
+    __shared__ int64_t sA, sB, sna, snb;
+    __shared__ int sfast;
+    const int tid = threadIdx.x;
+    const int64_t e0 = int64_t(blockIdx.x) * LM_T, e1 = dmin(e0 + LM_T, LP);
+    if (tid == 0) {
+        int64_t lo = 0, hi = nlong;
+        while (hi - lo > 1) {
+            const int64_t mid = (lo + hi) >> 1;
+            if (longO[mid] <= e0) lo = mid;
+            else hi = mid;
+        }
+        const int64_t O = longO[lo], P = longP[lo];
+        const int64_t a0 = ((e0 - O) / (2 * w)) * (2 * w);
+        const int64_t la = dmin(w, P - a0);
+        const int64_t lb = dmax(0, dmin(w, P - a0 - la));
+        const int64_t A0 = O + a0, B0 = A0 + la;
+        sfast = (e1 <= A0 + la + lb) ? 1 : 0;
+        if (sfast) {
+            auto split = [&](int64_t d) {
+                int64_t l2 = dmax(0, d - lb), h2 = dmin(d, la);
+                while (l2 < h2) {
+                    const int64_t mid = (l2 + h2) >> 1;
+                    if (Xc[A0 + mid] <= Xc[B0 + d - mid - 1]) l2 = mid + 1;
+                    else h2 = mid;
+                }
+                return l2;
+            };
+            const int64_t d0 = e0 - A0, d1 = e1 - A0;
+            const int64_t i0 = split(d0), i1 = split(d1);
+            sA = A0 + i0;
+            sB = B0 + (d0 - i0);
+            sna = i1 - i0;
+            snb = (d1 - i1) - (d0 - i0);
+        }
+    }
+    __syncthreads();
+    if (!sfast) {
+        const int64_t e = e0 + int64_t(tid) * LM_IPT;
+        long_merge_thread<NUM>(e, dmin(e + LM_IPT, e1), nlong, longO, longP, w, Xc, Xv, Yc, Yv);
+        return;
+    }
+    const int na = int(sna), nb = int(snb);
+    const int64_t gA = sA, gB = sB;
+    for (int x = tid; x < na + nb; x += LM_NT) {
+        const int64_t g = x < na ? gA + x : gB + (x - na);
+        sc[x] = Xc[g];
+        if (NUM) sv[x] = Xv[g];
+    }
+    __syncthreads();
+    const int d = min(tid * LM_IPT, na + nb);
+    int lo = max(0, d - nb), hi = min(d, na);
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (sc[mid] <= sc[na + d - mid - 1]) lo = mid + 1;
+        else hi = mid;
+    }
+    int ia = lo, ib = d - lo;
+    const int n = min(LM_IPT, na + nb - d);
+    const int64_t out = e0 + d;
+    for (int t = 0; t < n; ++t) {
+        const bool ta = ib >= nb || (ia < na && sc[ia] <= sc[na + ib]);
+        const int src = ta ? ia : na + ib;
+        Yc[out + t] = sc[src];
+        if (NUM) Yv[out + t] = sv[src];
+        ia += ta ? 1 : 0;
+        ib += ta ? 0 : 1;
     }
 }
 
@@ -780,8 +867,7 @@ msp_status run_long(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const
     int cur = 0;
     int64_t maxlong = h.maxP;
     for (int64_t w = GM_TL; w < maxlong; w *= 2) {
-        const int64_t threads = ceil_div(h.LP, 16);
-        long_merge_kernel<NUM><<<unsigned(ceil_div(threads, 256)), 256, 0, s>>>(
+        long_merge_kernel<NUM><<<unsigned(ceil_div(h.LP, LM_T)), LM_NT, 0, s>>>(
             h.LP, h.nlong, sw.longO, sw.longP, w, mw.Xc[cur], mw.Xv[cur], mw.Xc[cur ^ 1], mw.Xv[cur ^ 1]);
         st = last_launch("long_merge_kernel");
         if (st != MSP_OK) return st;
