@@ -119,3 +119,39 @@ def test_deterministic():
     _, _, v1, _ = run(A, A)
     _, _, v2, _ = run(A, A)
     assert np.array_equal(v1.view(np.uint8), v2.view(np.uint8))
+
+
+def check_sampled(A, B, rows, label):
+    """Full-size run in the bench's launch configuration; structure of the
+    whole C checked against its closed forms / totals, sampled rows element
+    by element against the oracle."""
+    rp, col, val, info = run(A, B)
+    off, wcol, wval, scale = oracle.spgemm_rows(A, B, rows)
+    for k, r in enumerate(rows):
+        a, b = int(rp[r]), int(rp[r + 1])
+        lo, hi = int(off[k]), int(off[k + 1])
+        assert b - a == hi - lo, f"{label}: row {r} length"
+        assert np.array_equal(col[a:b], wcol[lo:hi]), f"{label}: row {r} columns"
+        ok, msg = oracle.check_values(val[a:b], wval[lo:hi], scale[lo:hi], A.val.dtype)
+        assert ok, f"{label}: row {r}: {msg}"
+    return rp, info
+
+
+def test_c2_full_sampled():
+    """C2 A*A at full size (BJ:8): Nprods = 890^3, nnz(C) = 494^3."""
+    A = gen.config("C2", "random")
+    rows = np.unique(np.concatenate([np.arange(0, 200), np.linspace(0, A.m - 1, 300).astype(np.int64),
+                                     np.arange(A.m - 200, A.m)]))
+    rp, info = check_sampled(A, A, rows, "C2 full")
+    assert info.nprods == 890 ** 3 and int(rp[-1]) == 494 ** 3
+
+
+def test_c4_full_sampled():
+    """C4 A*A at full size (BJ:10), including the 1M-nnz dense row (long-row
+    path: chunk sorts + CTA merge passes) and empty rows."""
+    A = gen.config("C4", "int")
+    dense = int(np.argmax(np.diff(A.rp)))
+    rows = np.unique(np.concatenate([[dense, dense - 1, dense + 1], np.linspace(0, A.m - 1, 400).astype(np.int64),
+                                     np.arange(A.m - 50, A.m)]))
+    rp, info = check_sampled(A, A, rows, "C4 full")
+    assert info.long_rows >= 1 and int(rp[-1]) <= info.nprods
