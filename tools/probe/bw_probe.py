@@ -5,7 +5,13 @@ import json
 import os
 import torch
 
-L = ctypes.CDLL(os.path.join(os.path.dirname(os.path.abspath(__file__)), "bw_probe.so"))
+_HERE = os.path.dirname(os.path.abspath(__file__))
+if not os.path.exists(os.path.join(_HERE, "bw_probe.so")):
+    import subprocess
+    subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-shared",
+                           "-Xcompiler", "-fPIC", "-o", os.path.join(_HERE, "bw_probe.so"),
+                           os.path.join(_HERE, "bw_probe.cu")])
+L = ctypes.CDLL(os.path.join(_HERE, "bw_probe.so"))
 nbytes = 2 << 30
 a = torch.ones(nbytes // 4, dtype=torch.int32, device="cuda")
 out = torch.zeros(1, dtype=torch.int64, device="cuda")
