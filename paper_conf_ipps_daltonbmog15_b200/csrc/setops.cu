@@ -34,24 +34,26 @@ constexpr int SET_NT = 256;
 #endif
 constexpr int SET_IPT = MSP_SET_IPT;
 constexpr int SET_T = SET_NT * SET_IPT;  // merge items per tile (+1 for a starred cut)
+constexpr int SET_STEPS = SET_IPT + 1;  // register output slots per thread
 
 struct Cut {
     int64_t i, j;
 };
 
 // Balanced-path cut of diagonal d over key arrays A[0..na), B[0..nb)
-// (global or shared memory, any key type).  See partition_model.py
+// (global or shared memory, any key type; IT = index type, int64_t in global
+// memory, int inside a tile).  See partition_model.py
 // balanced_path_split_ranked for the reference statement of the rule.
-template <typename KT, class LA, class LB>
-__device__ __forceinline__ Cut balanced_cut(LA A, int64_t na, LB B, int64_t nb, int64_t d)
+template <typename KT, typename IT, class LA, class LB>
+__device__ __forceinline__ Cut balanced_cut(LA A, IT na, LB B, IT nb, IT d)
 {
-    int64_t lo = d > nb ? d - nb : 0, hi = d < na ? d : na;
+    IT lo = d > nb ? d - nb : 0, hi = d < na ? d : na;
     while (lo < hi) {  // merge path, A first on ties (Alg. 1)
-        const int64_t mid = (lo + hi) >> 1;
+        const IT mid = (lo + hi) >> 1;
         if (A(mid) <= B(d - mid - 1)) lo = mid + 1;
         else hi = mid;
     }
-    int64_t i = lo, j = d - lo;
+    const IT i = lo, j = d - lo;
     const bool hl = i > 0 || j > 0, hn = i < na || j < nb;
     if (!hl || !hn) return Cut{i, j};
     KT last = 0, next = ~KT(0);
@@ -61,28 +63,50 @@ __device__ __forceinline__ Cut balanced_cut(LA A, int64_t na, LB B, int64_t nb, 
     if (j < nb && B(j) < next) next = B(j);
     if (last != next) return Cut{i, j};  // the cut is between two keys
     const KT k = last;
-    auto lower = [&](auto X, int64_t l, int64_t h) {  // first index in [l, h) with X >= k
-        while (l < h) {
-            const int64_t m = (l + h) >> 1;
-            if (X(m) < k) l = m + 1;
-            else h = m;
+    // bounds of the run of key k around position x: galloping from x (runs
+    // are short next to the arrays), then bisection inside the bracket
+    auto lower = [&](auto X, IT x) {  // first index in [0, x] with X >= k (X(x) >= k or x == end)
+        IT step = 1, h = x;
+        while (h > 0 && X(h - 1) == k) {
+            const IT l = h > step ? h - step : 0;
+            if (X(l) < k) {
+                IT a = l + 1, b = h - 1;  // X(l) < k, X(b) == k: first >= k in (l, b]
+                while (a < b) {
+                    const IT m = (a + b) >> 1;
+                    if (X(m) < k) a = m + 1;
+                    else b = m;
+                }
+                return a;
+            }
+            h = l;
+            step <<= 1;
+        }
+        return h;
+    };
+    auto upper = [&](auto X, IT x, IT n) {  // first index in [x, n] with X > k
+        IT step = 1, l = x;
+        while (l < n && X(l) == k) {
+            const IT h = n - l > step ? l + step : n;
+            if (h == n || X(h) > k) {
+                IT a = l + 1, b = h;  // X(l) == k, X(h) > k (or h == n): first > k in (l, h]
+                while (a < b) {
+                    const IT m = (a + b) >> 1;
+                    if (X(m) <= k) a = m + 1;
+                    else b = m;
+                }
+                return a;
+            }
+            l = h;  // X(h) == k
+            step <<= 1;
         }
         return l;
     };
-    auto upper = [&](auto X, int64_t l, int64_t h) {  // first index in [l, h) with X > k
-        while (l < h) {
-            const int64_t m = (l + h) >> 1;
-            if (X(m) <= k) l = m + 1;
-            else h = m;
-        }
-        return l;
-    };
-    const int64_t a_lo = lower(A, 0, i), a_hi = upper(A, i, na);
-    const int64_t b_lo = lower(B, 0, j), b_hi = upper(B, j, nb);
-    const int64_t ca = a_hi - a_lo, cb = b_hi - b_lo;
-    const int64_t p = (i - a_lo) + (j - b_lo);  // items of key k before the cut
-    const int64_t mm = ca < cb ? ca : cb;
-    int64_t ia, ib;
+    const IT a_lo = lower(A, i), a_hi = upper(A, i, na);
+    const IT b_lo = lower(B, j), b_hi = upper(B, j, nb);
+    const IT ca = a_hi - a_lo, cb = b_hi - b_lo;
+    const IT p = (i - a_lo) + (j - b_lo);  // items of key k before the cut
+    const IT mm = ca < cb ? ca : cb;
+    IT ia, ib;
     if (p <= 2 * mm) {
         ia = (p + 1) >> 1;
         ib = p >> 1;
@@ -105,7 +129,7 @@ __global__ void set_partition_kernel(const KT *__restrict__ A, int64_t na, const
     for (int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; k <= ntiles;
          k += int64_t(gridDim.x) * blockDim.x) {
         const int64_t d = k * SET_T < total ? k * SET_T : total;
-        cuts[k] = balanced_cut<KT>([&](int64_t x) { return A[x]; }, na, [&](int64_t x) { return B[x]; }, nb, d);
+        cuts[k] = balanced_cut<KT, int64_t>([&](int64_t x) { return A[x]; }, na, [&](int64_t x) { return B[x]; }, nb, d);
     }
 }
 
@@ -144,19 +168,21 @@ set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t n
     const int tile = S.tile;
     const Cut c0 = cuts[tile], c1 = cuts[tile + 1];
     const int la = int(c1.i - c0.i), lb = int(c1.j - c0.j);
+    // stage both windows with asynchronous element copies (LDGSTS): every
+    // copy of the tile is in flight at once, no register round trip
     for (int x = tid; x < la; x += SET_NT) {
-        S.ka[x] = A[c0.i + x];
-        if constexpr (VB > 0) S.va[x] = static_cast<const VT *>(Av)[c0.i + x];
+        cp_async<sizeof(KT)>(&S.ka[x], &A[c0.i + x]);
+        if constexpr (VB > 0) cp_async<VB>(&S.va[x], static_cast<const VT *>(Av) + c0.i + x);
     }
     for (int x = tid; x < lb; x += SET_NT) {
-        S.kb[x] = B[c0.j + x];
-        if constexpr (VB > 0) S.vb[x] = static_cast<const VT *>(Bv)[c0.j + x];
+        cp_async<sizeof(KT)>(&S.kb[x], &B[c0.j + x]);
+        if constexpr (VB > 0) cp_async<VB>(&S.vb[x], static_cast<const VT *>(Bv) + c0.j + x);
     }
+    cp_async_wait_all();
     __syncthreads();
     {  // this thread's cut inside the tile (windows clipped to the tile: consistent, R4)
         const int d = min(tid * SET_IPT, la + lb);
-        const Cut c = balanced_cut<KT>([&](int64_t x) { return S.ka[x]; }, la, [&](int64_t x) { return S.kb[x]; },
-                                       lb, d);
+        const Cut c = balanced_cut<KT, int>([&](int x) { return S.ka[x]; }, la, [&](int x) { return S.kb[x]; }, lb, d);
         S.cut_i[tid] = int(c.i);
         S.cut_j[tid] = int(c.j);
         if (tid == 0) {
@@ -168,6 +194,10 @@ set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t n
     // a starred cut may pass the next thread's nominal diagonal: clamp (monotone)
     int ia0 = S.cut_i[tid], ib0 = S.cut_j[tid];
     int ia1 = max(S.cut_i[tid + 1], ia0), ib1 = max(S.cut_j[tid + 1], ib0);
+    // A thread's window holds <= SET_IPT + 1 items (its end cut may be starred)
+    // and every walk step consumes >= 1 of them, so SET_STEPS register slots
+    // hold its outputs; a CTA where that fails takes the two-walk path.
+    const bool regs = __syncthreads_and((ia1 - ia0) + (ib1 - ib0) <= SET_STEPS);
     auto walk = [&](auto &&emit) {
         int ia = ia0, ib = ib0;
         while (ia < ia1 || ib < ib1) {
@@ -185,38 +215,109 @@ set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t n
             }
         }
     };
+    KT rk[SET_STEPS];
+    VT rv[VB > 0 ? SET_STEPS : 1];
+    unsigned emitted = 0;
     int cnt = 0;
-    walk([&](bool, int) { ++cnt; });
+    if (regs) {  // one walk, outputs kept in registers (static slot per step)
+        int ia = ia0, ib = ib0;
+#pragma unroll
+        for (int s = 0; s < SET_STEPS; ++s) {
+            const bool ra = ia < ia1, rb = ib < ib1;
+            if (ra || rb) {
+                const KT ka = ra ? S.ka[ia] : KT(0), kb = rb ? S.kb[ib] : KT(0);
+                bool e, fromA;
+                if (ra && (!rb || ka < kb)) {
+                    e = EA, fromA = true;
+                } else if (rb && (!ra || kb < ka)) {
+                    e = EB, fromA = false;
+                } else {  // matched key-rank pair: A's copy
+                    e = EM, fromA = true;
+                    ++ib;
+                }
+                rk[s] = fromA ? ka : kb;
+                if constexpr (VB > 0) rv[s] = fromA ? S.va[ia] : S.vb[ib];
+                if (fromA) ++ia;
+                else ++ib;
+                if (e) {
+                    emitted |= 1u << s;
+                    ++cnt;
+                }
+            }
+        }
+    } else {
+        walk([&](bool, int) { ++cnt; });
+    }
     int tot;
     const int off = block_exclusive_sum<int, SET_NT / 32>(cnt, S.wsum, 1, &tot);
-    if (tid == 0) {  // decoupled look-back over the tiles
+    // past the scan's barrier every thread has finished reading the windows:
+    // the register path stages the tile's outputs over ka / va
+    if (regs) {
+        int p = off;
+#pragma unroll
+        for (int s = 0; s < SET_STEPS; ++s) {
+            if (emitted & (1u << s)) {
+                S.ka[p] = rk[s];
+                if constexpr (VB > 0) S.va[p] = rv[s];
+                ++p;
+            }
+        }
+    }
+    if (tid < 32) {  // decoupled look-back over the tiles (warp 0, 32 predecessors per round)
+        const int lane = tid;
         int64_t excl = 0;
         if (tile == 0) {
-            __threadfence();
-            atomicExch(reinterpret_cast<unsigned long long *>(&states[0]), (unsigned long long)(ST_PRE | uint64_t(tot)));
-        } else {
-            atomicExch(reinterpret_cast<unsigned long long *>(&states[tile]), (unsigned long long)(ST_AGG | uint64_t(tot)));
-            for (int k = tile - 1; k >= 0;) {
-                const uint64_t st = *reinterpret_cast<volatile uint64_t *>(&states[k]);
-                if ((st & ~ST_VAL) == 0) continue;  // predecessor not published yet
-                excl += int64_t(st & ST_VAL);
-                if (st & ST_PRE) break;
-                --k;
+            if (lane == 0) {
+                __threadfence();
+                atomicExch(reinterpret_cast<unsigned long long *>(&states[0]),
+                           (unsigned long long)(ST_PRE | uint64_t(tot)));
             }
-            __threadfence();
-            atomicExch(reinterpret_cast<unsigned long long *>(&states[tile]),
-                       (unsigned long long)(ST_PRE | uint64_t(excl + tot)));
+        } else {
+            if (lane == 0)
+                atomicExch(reinterpret_cast<unsigned long long *>(&states[tile]),
+                           (unsigned long long)(ST_AGG | uint64_t(tot)));
+            for (int pos = tile - 1;; pos -= 32) {
+                const int k = pos - lane;
+                uint64_t st = ST_PRE;  // virtual prefix 0 before tile 0
+                if (k >= 0) {
+                    do {
+                        st = *reinterpret_cast<volatile uint64_t *>(&states[k]);
+                    } while ((st & ~ST_VAL) == 0);  // predecessor not published yet
+                }
+                const unsigned pre = __ballot_sync(0xffffffffu, (st & ST_PRE) != 0);
+                const int stop = pre ? __ffs(pre) - 1 : 32;  // nearest predecessor with a prefix
+                int64_t v = lane <= stop ? int64_t(st & ST_VAL) : 0;
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+                excl += v;
+                if (pre) break;
+            }
+            if (lane == 0) {
+                __threadfence();
+                atomicExch(reinterpret_cast<unsigned long long *>(&states[tile]),
+                           (unsigned long long)(ST_PRE | uint64_t(excl + tot)));
+            }
         }
-        S.base = excl;
-        if (tile == ntiles - 1) *nC = excl + tot;
+        if (lane == 0) {
+            S.base = excl;
+            if (tile == ntiles - 1) *nC = excl + tot;
+        }
     }
     __syncthreads();
-    int64_t pos = S.base + off;
-    walk([&](bool fromA, int x) {
-        C[pos] = fromA ? S.ka[x] : S.kb[x];
-        if constexpr (VB > 0) static_cast<VT *>(Cv)[pos] = fromA ? S.va[x] : S.vb[x];
-        ++pos;
-    });
+    const int64_t base = S.base;
+    if (regs) {  // coalesced store of the staged run
+        for (int x = tid; x < tot; x += SET_NT) {
+            C[base + x] = S.ka[x];
+            if constexpr (VB > 0) static_cast<VT *>(Cv)[base + x] = S.va[x];
+        }
+    } else {
+        int64_t pos = base + off;
+        walk([&](bool fromA, int x) {
+            C[pos] = fromA ? S.ka[x] : S.kb[x];
+            if constexpr (VB > 0) static_cast<VT *>(Cv)[pos] = fromA ? S.va[x] : S.vb[x];
+            ++pos;
+        });
+    }
 }
 
 struct SetWs {
