@@ -45,6 +45,7 @@ constexpr int ADD_NT = 256;
 #endif
 constexpr int ADD_IPT = MSP_ADD_IPT;  // merge items per thread
 constexpr int ADD_T = ADD_NT * ADD_IPT;  // merge items per tile
+constexpr int ADD_STEPS = ADD_IPT + 1;   // register output slots per thread (fill)
 
 struct Split {
     int32_t r, a, b;  // row (row-end items consumed), A index, B index (global)
@@ -304,20 +305,72 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
     } else {
         int32_t *ocol = reinterpret_cast<int32_t *>(smem_raw + L::O_OFF);
         V *oval = reinterpret_cast<V *>(smem_raw + L::O_OFF + 4 * ADD_T);
+        // A thread's path holds (end - beg) items over the three coordinates
+        // and every step consumes >= 1 of them: when all fit ADD_STEPS static
+        // register slots, ONE walk forms the outputs (CTA-uniform choice;
+        // otherwise count, scan, walk again).
+        const int nit = (end.r - beg.r) + (end.a - beg.a) + (end.b - beg.b);
+        const bool regs = __syncthreads_and(nit <= ADD_STEPS);
         int cnt = 0;
-        walk([&](int, int, int) { ++cnt; }, [&](int) {});
+        int rc[ADD_STEPS];
+        V rv[ADD_STEPS];
+        unsigned em = 0;
+        if (regs) {
+            int r = beg.r, ia = beg.a, ib = beg.b;
+            int ah = (r < m) ? a_hi(r) : nA, bh = (r < m) ? b_hi(r) : nB;
+#pragma unroll
+            for (int st = 0; st < ADD_STEPS; ++st) {
+                if (r != end.r || ia != end.a || ib != end.b) {
+                    const bool ra = ia < ah, rb = ib < bh;
+                    if (!ra && !rb) {  // row-end item
+                        ++r;
+                        if (r < m) {
+                            ah = a_hi(r);
+                            bh = b_hi(r);
+                        }
+                    } else {
+                        const int ca = ra ? acs[ia] : INT_MAX, cb = rb ? bcs[ib] : INT_MAX;
+                        if (ca <= cb) {
+                            rc[st] = ca;
+                            rv[st] = (ca == cb) ? avs[ia] + bvs[ib] : avs[ia];  // one rounding, A first (Alg. 1)
+                            ib += (ca == cb);
+                            ++ia;
+                        } else {
+                            rc[st] = cb;
+                            rv[st] = bvs[ib];
+                            ++ib;
+                        }
+                        em |= 1u << st;
+                        ++cnt;
+                    }
+                }
+            }
+        } else {
+            walk([&](int, int, int) { ++cnt; }, [&](int) {});
+        }
         int tot;
         int o = block_exclusive_sum<int, ADD_NT / 32>(cnt, S_wsum, 0, &tot);
-        walk(
-            [&](int c, int ia, int ib) {
-                V v;
-                if (ia >= 0 && ib >= 0) v = avs[ia] + bvs[ib];  // one rounding, A first (Alg. 1)
-                else v = (ia >= 0) ? avs[ia] : bvs[ib];
-                ocol[o] = c;
-                oval[o] = v;
-                ++o;
-            },
-            [&](int) {});
+        if (regs) {
+#pragma unroll
+            for (int st = 0; st < ADD_STEPS; ++st) {
+                if (em & (1u << st)) {
+                    ocol[o] = rc[st];
+                    oval[o] = rv[st];
+                    ++o;
+                }
+            }
+        } else {
+            walk(
+                [&](int c, int ia, int ib) {
+                    V v;
+                    if (ia >= 0 && ib >= 0) v = avs[ia] + bvs[ib];  // one rounding, A first (Alg. 1)
+                    else v = (ia >= 0) ? avs[ia] : bvs[ib];
+                    ocol[o] = c;
+                    oval[o] = v;
+                    ++o;
+                },
+                [&](int) {});
+        }
         __syncthreads();
         // the tile's run of C is contiguous: coalesced stores
         const int64_t base = tile_off[k];
