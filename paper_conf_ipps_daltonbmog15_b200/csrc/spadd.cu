@@ -118,8 +118,11 @@ struct AddLayout {
     static constexpr int VBYTES = FILL ? int(sizeof(V)) * ADD_T + 2 * 32 : 0;
     static constexpr int OBYTES = FILL ? (4 + int(sizeof(V))) * ADD_T : 0;
     static constexpr int V_OFF = IBYTES;
-    static constexpr int O_OFF = V_OFF + VBYTES;
-    static constexpr int ST_OFF = (O_OFF + OBYTES + 15) / 16 * 16;
+    // the output run overlays the input windows: it is written only after
+    // the scan barrier, when every thread has finished reading them
+    static constexpr int O_OFF = 0;
+    static_assert(OBYTES <= V_OFF + VBYTES, "output run must fit over the input windows");
+    static constexpr int ST_OFF = (V_OFF + VBYTES + 15) / 16 * 16;
     static constexpr int WS_OFF = ST_OFF + int(sizeof(Split)) * (ADD_NT + 1);
     static constexpr int BAR_OFF = (WS_OFF + 4 * (ADD_NT / 32) + 15) / 16 * 16;
     static constexpr int BYTES = BAR_OFF + 16;
@@ -310,7 +313,11 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
         // register slots, ONE walk forms the outputs (CTA-uniform choice;
         // otherwise count, scan, walk again).
         const int nit = (end.r - beg.r) + (end.a - beg.a) + (end.b - beg.b);
+#ifdef MSP_ADD_FORCE_WALK2  // test build: exercise the fallback path
+        const bool regs = __syncthreads_and(nit < 0);
+#else
         const bool regs = __syncthreads_and(nit <= ADD_STEPS);
+#endif
         int cnt = 0;
         int rc[ADD_STEPS];
         V rv[ADD_STEPS];
@@ -359,24 +366,27 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
                     ++o;
                 }
             }
-        } else {
+        } else {  // fallback: the windows are still being read, store straight to C
+            int64_t p = tile_off[k] + o;
             walk(
                 [&](int c, int ia, int ib) {
                     V v;
                     if (ia >= 0 && ib >= 0) v = avs[ia] + bvs[ib];  // one rounding, A first (Alg. 1)
                     else v = (ia >= 0) ? avs[ia] : bvs[ib];
-                    ocol[o] = c;
-                    oval[o] = v;
-                    ++o;
+                    Ccol[p] = c;
+                    Cval[p] = v;
+                    ++p;
                 },
                 [&](int) {});
         }
-        __syncthreads();
-        // the tile's run of C is contiguous: coalesced stores
-        const int64_t base = tile_off[k];
-        for (int i = tid; i < tot; i += ADD_NT) {
-            Ccol[base + i] = ocol[i];
-            Cval[base + i] = oval[i];
+        if (regs) {
+            __syncthreads();
+            // the tile's run of C is contiguous: coalesced stores
+            const int64_t base = tile_off[k];
+            for (int i = tid; i < tot; i += ADD_NT) {
+                Ccol[base + i] = ocol[i];
+                Cval[base + i] = oval[i];
+            }
         }
     }
 }
