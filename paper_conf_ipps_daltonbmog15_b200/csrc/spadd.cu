@@ -41,7 +41,8 @@ namespace {
 
 constexpr int ADD_NT = 256;
 #ifndef MSP_ADD_IPT
-#define MSP_ADD_IPT 12  // measured on B200: C3 A+A^T 1.96 ms at 8, 1.71 at 12, 1.83 at 16
+#define MSP_ADD_IPT 14  // measured on B200 (one-walk fill, 53-66 KB smem): C3 A+A^T 1.85 ms at 8, 1.42 at 12,
+                        // 1.30 at 14, 1.31 at 16, 1.23 at 20; C2 0.47-0.49 ms at 12-20
 #endif
 constexpr int ADD_IPT = MSP_ADD_IPT;  // merge items per thread
 constexpr int ADD_T = ADD_NT * ADD_IPT;  // merge items per tile
