@@ -216,7 +216,11 @@ set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t n
     // A thread's window holds <= SET_IPT + 1 items (its end cut may be starred)
     // and every walk step consumes >= 1 of them, so SET_STEPS register slots
     // hold its outputs; a CTA where that fails takes the two-walk path.
+#ifdef MSP_SET_FORCE_WALK2  // test build: exercise the two-walk path
+    const bool regs = __syncthreads_and(ia1 < ia0);
+#else
     const bool regs = __syncthreads_and((ia1 - ia0) + (ib1 - ib0) <= SET_STEPS);
+#endif
     auto walk = [&](auto &&emit) {
         int ia = ia0, ib = ib0;
         while (ia < ia1 || ib < ib1) {
@@ -270,18 +274,22 @@ set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t n
     int tot;
     const int off = block_exclusive_sum<int, SET_NT / 32>(cnt, S.wsum, 1, &tot);
     // past the scan's barrier every thread has finished reading the windows:
-    // the register path stages the tile's outputs over ka / va
-    if (regs) {
-        int p = off;
+    // the register path stages the tile's outputs over ka / va (warp 0 after
+    // the look-back, so the tile's aggregate is published right after the scan)
+    auto stage_out = [&]() {
+        if (regs) {
+            int p = off;
 #pragma unroll
-        for (int s = 0; s < SET_STEPS; ++s) {
-            if (emitted & (1u << s)) {
-                S.ka[p] = rk[s];
-                if constexpr (VB > 0) S.va[p] = rv[s];
-                ++p;
+            for (int s = 0; s < SET_STEPS; ++s) {
+                if (emitted & (1u << s)) {
+                    S.ka[p] = rk[s];
+                    if constexpr (VB > 0) S.va[p] = rv[s];
+                    ++p;
+                }
             }
         }
-    }
+    };
+    if (tid >= 32) stage_out();
     if (tid < 32) {  // decoupled look-back over the tiles (warp 0, 32 predecessors per round)
         const int lane = tid;
         int64_t excl = 0;
@@ -319,6 +327,7 @@ set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t n
             S.base = excl;
             if (tile == ntiles - 1) *nC = excl + tot;
         }
+        stage_out();
     }
     __syncthreads();
     const int64_t base = S.base;
