@@ -446,9 +446,22 @@ msp_status set_op_run(int op, const void *A, const void *Av, int64_t na, const v
     st = (key_bytes == 4) ? launch_kv<uint32_t>(op, val_bytes, A, Av, na, B, Bv, nb, w, C, Cv, s)
                           : launch_kv<uint64_t>(op, val_bytes, A, Av, na, B, Bv, nb, w, C, Cv, s);
     if (st != MSP_OK) return st;
-    st = cuda_check(cudaMemcpyAsync(nC_host, w.nC, sizeof(int64_t), cudaMemcpyDeviceToHost, s), "set op: size");
+    // the result size comes back through a pinned word (a pageable
+    // destination would stage the 8-byte copy through a driver buffer)
+    static thread_local int64_t *pinned = nullptr;
+    if (!pinned) {
+        st = cuda_check(cudaMallocHost(reinterpret_cast<void **>(&pinned), sizeof(int64_t)), "set op: pinned size");
+        if (st != MSP_OK) {
+            pinned = nullptr;
+            return st;
+        }
+    }
+    st = cuda_check(cudaMemcpyAsync(pinned, w.nC, sizeof(int64_t), cudaMemcpyDeviceToHost, s), "set op: size");
     if (st != MSP_OK) return st;
-    return cuda_check(cudaStreamSynchronize(s), "set op: sync");
+    st = cuda_check(cudaStreamSynchronize(s), "set op: sync");
+    if (st != MSP_OK) return st;
+    *nC_host = *pinned;
+    return MSP_OK;
 }
 
 }  // namespace msp
