@@ -182,9 +182,13 @@ set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t n
     extern __shared__ __align__(16) char smem_raw[];
     SetSmem<KT, VB> &S = *reinterpret_cast<SetSmem<KT, VB> *>(smem_raw);
     const int tid = threadIdx.x;
+#ifdef MSP_SET_BLOCKID_TILES  // experiment: tile = blockIdx.x (relies on in-order CTA dispatch)
+    const int tile = int(blockIdx.x);
+#else
     if (tid == 0) S.tile = int(atomicAdd(ticket, 1u));  // tiles in claim order: look-back never waits on an unstarted tile
     __syncthreads();
     const int tile = S.tile;
+#endif
     const Cut c0 = cuts[tile], c1 = cuts[tile + 1];
     const int la = int(c1.i - c0.i), lb = int(c1.j - c0.j);
     // stage both windows with asynchronous element copies (LDGSTS): every
