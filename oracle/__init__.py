@@ -209,7 +209,12 @@ def check_values(got: np.ndarray, want: np.ndarray, scale: np.ndarray, dtype) ->
     gn, wn = np.isnan(g), np.isnan(w)
     if not np.array_equal(gn, wn):
         return False, "NaN positions differ"
-    ok = ~gn
+    # an infinity propagates (Z19): where either side is infinite both must be
+    # the same infinity (|inf - -inf| <= tau * inf would otherwise pass)
+    inf = (np.isinf(g) | np.isinf(w)) & ~gn
+    if np.any(g[inf] != w[inf]):
+        return False, "infinities differ"
+    ok = ~gn & ~inf
     err = np.abs(g[ok] - w[ok])
     # fp32 results are rounded once from an fp64 accumulator on both sides
     # (Z4); a one-ulp difference of the stored value is <= 2^-23 |y| <=
