@@ -57,7 +57,7 @@
 extern "C" {
 #endif
 
-#define MSP_VERSION 1
+#define MSP_VERSION 2  /* 2: msp_spgemm_info passed to symbolic / numeric */
 
 typedef enum {
     MSP_OK = 0,
@@ -140,21 +140,25 @@ msp_status msp_spadd_numeric(const msp_csr *A, const msp_csr *B, const int32_t *
  * Setup: S = exclusive prefix sum (int64) of the B row lengths
  * referenced by A's column indices, Nprods = S[nnzA], the COO row of every
  * A nonzero, and the classification of rows whose product count exceeds
- * one tile.  Returns the sizes in *info_host and synchronises.
+ * one tile.  Returns the sizes in *info_host; synchronises the stream once.
  * Symbolic: products are partitioned into tiles by a merge-path search over
  * (S, product index) (reading Z7), expanded, sorted by
  * (row, col) with a block merge sort and compressed; rows that straddle a
  * tile boundary and rows longer than a tile are completed by a second pass
  * (the paper's global phase).  Writes C_row_offsets and
- * *nnzC_host; synchronises.  MSP_ERR_OVERFLOW if nnz(C) > INT32_MAX.
- * The symbolic pass keeps every tile's sorting permutation in main_ws
- * (2 bytes per tile slot, as the paper stores the CTA sort's permutation,
- * P:1140-1175).
+ * *nnzC_host and records the largest tile row span in info_host (in/out:
+ * pass the struct setup filled); synchronises the stream twice (the tile
+ * key width depends on that span; nnz(C)).  MSP_ERR_OVERFLOW if nnz(C) >
+ * INT32_MAX.  The symbolic pass keeps every tile's sorting permutation in
+ * main_ws (2 bytes per tile slot, as the paper stores the CTA sort's
+ * permutation).
  * Numeric: re-expands the products with values, applies the stored
  * permutation (no second sort) and compresses; the long-row pass is repeated
  * with values.  Writes C_col_idx / C_vals; fp64 accumulation in a fixed,
- * deterministic order.  Must follow msp_spgemm_symbolic on the same main_ws
- * with A and B unchanged.  Async.
+ * deterministic order.  Must follow msp_spgemm_symbolic on the same
+ * setup_ws / main_ws, with A and B unchanged, and get the info_host that
+ * symbolic updated (MSP_ERR_ARG if max_tile_span is unset).  Async: no
+ * synchronisation, every size comes from info_host.
  * setup_ws: msp_spgemm_setup_workspace() bytes; main_ws: info.main_ws_bytes.
  * ------------------------------------------------------------------------ */
 typedef struct {
@@ -164,6 +168,9 @@ typedef struct {
     int64_t long_products;   /* products in those rows */
     int64_t max_row_products;
     int64_t main_ws_bytes;   /* size of the main workspace */
+    int64_t long_chunks;     /* sorted chunks of the long-row pass */
+    int64_t max_tile_span;   /* largest row span of a product tile: -1 after
+                                setup, set by symbolic (picks the key width) */
 } msp_spgemm_info;
 
 msp_status msp_spgemm_setup_workspace(const msp_csr *A, const msp_csr *B, size_t *bytes);
@@ -171,11 +178,12 @@ msp_status msp_spgemm_setup(const msp_csr *A, const msp_csr *B, void *setup_ws,
                             size_t setup_ws_bytes, msp_spgemm_info *info_host, void *stream);
 msp_status msp_spgemm_symbolic(const msp_csr *A, const msp_csr *B, const void *setup_ws,
                                size_t setup_ws_bytes, void *main_ws, size_t main_ws_bytes,
-                               int32_t *C_row_offsets, int64_t *nnzC_host, void *stream);
+                               msp_spgemm_info *info_host, int32_t *C_row_offsets,
+                               int64_t *nnzC_host, void *stream);
 msp_status msp_spgemm_numeric(const msp_csr *A, const msp_csr *B, const void *setup_ws,
                               size_t setup_ws_bytes, void *main_ws, size_t main_ws_bytes,
-                              const int32_t *C_row_offsets, int32_t *C_col_idx, void *C_vals,
-                              void *stream);
+                              const msp_spgemm_info *info_host, const int32_t *C_row_offsets,
+                              int32_t *C_col_idx, void *C_vals, void *stream);
 
 /* ------------------------------------------------------------------------
  * Input validation (the CSR contract of P:316-322).
@@ -204,8 +212,11 @@ msp_status msp_csr_check(const msp_csr *A, int require_sorted_unique, int32_t *f
  * must be at least nA + nB (union, symmetric difference), min(nA, nB)
  * (intersection) or nA (difference), else MSP_ERR_SHAPE.  *nC_host receives
  * the result size.  ws: msp_set_op_workspace() bytes, caller-owned.
- * Synchronises the stream (returns the size).  Unsorted input gives an
- * unspecified (but memory-safe) result.
+ * Synchronises the stream (returns the size).  Keys not sorted ascending
+ * (as unsigned integers; a signed tensor holding negatives is not) give
+ * MSP_ERR_INPUT: every tile checks its windows while staging them, reads
+ * and writes stay inside the given arrays and C_capacity, and the contents
+ * of C are then unspecified.
  * ------------------------------------------------------------------------ */
 typedef enum {
     MSP_SET_UNION = 0,

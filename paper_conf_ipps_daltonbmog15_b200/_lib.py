@@ -45,7 +45,8 @@ class msp_csr(ctypes.Structure):
 class msp_spgemm_info(ctypes.Structure):
     _fields_ = [("nprods", ctypes.c_int64), ("ntiles", ctypes.c_int64), ("long_rows", ctypes.c_int64),
                 ("long_products", ctypes.c_int64), ("max_row_products", ctypes.c_int64),
-                ("main_ws_bytes", ctypes.c_int64)]
+                ("main_ws_bytes", ctypes.c_int64), ("long_chunks", ctypes.c_int64),
+                ("max_tile_span", ctypes.c_int64)]
 
 
 _P = ctypes.POINTER
@@ -67,8 +68,10 @@ _SIGS = {
     "msp_spadd_numeric": (ctypes.c_int, [_csr_p, _csr_p, _vp, _vp, _vp, _vp, _sz, _vp]),
     "msp_spgemm_setup_workspace": (ctypes.c_int, [_csr_p, _csr_p, _P(_sz)]),
     "msp_spgemm_setup": (ctypes.c_int, [_csr_p, _csr_p, _vp, _sz, _P(msp_spgemm_info), _vp]),
-    "msp_spgemm_symbolic": (ctypes.c_int, [_csr_p, _csr_p, _vp, _sz, _vp, _sz, _vp, _P(_i64), _vp]),
-    "msp_spgemm_numeric": (ctypes.c_int, [_csr_p, _csr_p, _vp, _sz, _vp, _sz, _vp, _vp, _vp, _vp]),
+    "msp_spgemm_symbolic": (ctypes.c_int, [_csr_p, _csr_p, _vp, _sz, _vp, _sz, _P(msp_spgemm_info), _vp, _P(_i64),
+                                           _vp]),
+    "msp_spgemm_numeric": (ctypes.c_int, [_csr_p, _csr_p, _vp, _sz, _vp, _sz, _P(msp_spgemm_info), _vp, _vp, _vp,
+                                          _vp]),
     "msp_csr_check": (ctypes.c_int, [_csr_p, ctypes.c_int, _P(_i32), _vp, _sz, _vp]),
     "msp_row_split": (ctypes.c_int, [_vp, _i32, _i32, _vp]),
     "msp_rebase_offsets": (ctypes.c_int, [_vp, _vp, _i64, _i64, _vp]),

@@ -56,6 +56,43 @@ int sm_count()
     return cache[dev];
 }
 
+// Large-shared-memory opt-in, once per (device, kernel): the attribute is a
+// per-device property, so a process driving several GPUs sets it on each.
+// Returns the occupancy (resident CTAs per SM) when `threads` > 0.
+msp_status set_smem_attr(const void *func, int smem_bytes, const char *where, int threads, int *occ)
+{
+    struct Entry {
+        int dev;
+        const void *func;
+        int occ;
+    };
+    static std::mutex mu;
+    static Entry table[1024];
+    static int n = 0;
+    int dev = 0;
+    msp_status st = cuda_check(cudaGetDevice(&dev), where);
+    if (st != MSP_OK) return st;
+    std::lock_guard<std::mutex> lk(mu);
+    for (int i = 0; i < n; ++i)
+        if (table[i].dev == dev && table[i].func == func) {
+            if (occ) *occ = table[i].occ;
+            return MSP_OK;
+        }
+    st = cuda_check(cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes), where);
+    if (st != MSP_OK) return st;
+    int o = 1;
+    if (threads > 0) {
+        st = cuda_check(cudaFuncSetAttribute(func, cudaFuncAttributePreferredSharedMemoryCarveout, 100), where);
+        if (st != MSP_OK) return st;
+        st = cuda_check(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, func, threads, size_t(smem_bytes)), where);
+        if (st != MSP_OK) return st;
+        if (o < 1) o = 1;
+    }
+    if (n < 1024) table[n++] = Entry{dev, func, o};
+    if (occ) *occ = o;
+    return MSP_OK;
+}
+
 }  // namespace msp
 
 using namespace msp;
@@ -231,27 +268,29 @@ msp_status msp_spgemm_setup(const msp_csr *A, const msp_csr *B, void *setup_ws, 
 }
 
 msp_status msp_spgemm_symbolic(const msp_csr *A, const msp_csr *B, const void *setup_ws, size_t setup_ws_bytes,
-                               void *main_ws, size_t main_ws_bytes, int32_t *C_row_offsets, int64_t *nnzC_host,
-                               void *stream)
+                               void *main_ws, size_t main_ws_bytes, msp_spgemm_info *info_host,
+                               int32_t *C_row_offsets, int64_t *nnzC_host, void *stream)
 {
     clear_error();
     msp_status st = check_pair_mul(A, B);
     if (st != MSP_OK) return st;
-    if (!setup_ws || !main_ws || !C_row_offsets || !nnzC_host) return MSP_ERR_ARG;
-    return spgemm_symbolic_run(A, B, setup_ws, setup_ws_bytes, main_ws, main_ws_bytes, C_row_offsets, nnzC_host,
-                               as_stream(stream));
+    if (!setup_ws || !main_ws || !info_host || !C_row_offsets || !nnzC_host) return MSP_ERR_ARG;
+    if (main_ws_bytes < size_t(info_host->main_ws_bytes)) return MSP_ERR_WORKSPACE;
+    return spgemm_symbolic_run(A, B, setup_ws, setup_ws_bytes, main_ws, main_ws_bytes, info_host, C_row_offsets,
+                               nnzC_host, as_stream(stream));
 }
 
 msp_status msp_spgemm_numeric(const msp_csr *A, const msp_csr *B, const void *setup_ws, size_t setup_ws_bytes,
-                              void *main_ws, size_t main_ws_bytes, const int32_t *C_row_offsets,
-                              int32_t *C_col_idx, void *C_vals, void *stream)
+                              void *main_ws, size_t main_ws_bytes, const msp_spgemm_info *info_host,
+                              const int32_t *C_row_offsets, int32_t *C_col_idx, void *C_vals, void *stream)
 {
     clear_error();
     msp_status st = check_pair_mul(A, B);
     if (st != MSP_OK) return st;
-    if (!setup_ws || !main_ws || !C_row_offsets) return MSP_ERR_ARG;
-    return spgemm_numeric_run(A, B, setup_ws, setup_ws_bytes, main_ws, main_ws_bytes, C_row_offsets, C_col_idx,
-                              C_vals, as_stream(stream));
+    if (!setup_ws || !main_ws || !info_host || !C_row_offsets) return MSP_ERR_ARG;
+    if (main_ws_bytes < size_t(info_host->main_ws_bytes)) return MSP_ERR_WORKSPACE;
+    return spgemm_numeric_run(A, B, setup_ws, setup_ws_bytes, main_ws, main_ws_bytes, info_host, C_row_offsets,
+                              C_col_idx, C_vals, as_stream(stream));
 }
 
 // ------------------------------------------------------------------ misc
@@ -338,7 +377,8 @@ msp_status msp_set_operation(msp_set_op op, const void *A_keys, const void *A_va
         return MSP_ERR_ARG;
     }
     if (!ws && nA + nB > 0) return MSP_ERR_ARG;
-    return set_op_run(int(op), A_keys, A_vals, nA, B_keys, B_vals, nB, key_bytes, val_bytes, C_keys, C_vals, nC_host,
+    return set_op_run(int(op), A_keys, A_vals, nA, B_keys, B_vals, nB, key_bytes, val_bytes, C_keys, C_vals, C_capacity,
+                      nC_host,
                       ws, ws_bytes, as_stream(stream));
 }
 

@@ -20,7 +20,9 @@ __global__ void csr_check_kernel(int32_t m, int32_t ncols, int64_t nnz, const in
     }
     for (int64_t r = warp; r < m; r += nwarps) {
         const int32_t a = rp[r], b = rp[r + 1];
-        if (b < a) {
+        // a malformed row is flagged and skipped before col is touched, so the
+        // validator never reads outside col[0, nnz) on the input it rejects
+        if (a < 0 || b < a || int64_t(b) > nnz) {
             f |= 1;
             continue;
         }

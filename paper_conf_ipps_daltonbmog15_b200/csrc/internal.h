@@ -20,6 +20,9 @@ int sm_count();
 msp_status cuda_check(cudaError_t e, const char *where);
 msp_status last_launch(const char *where);  // also counts the launch
 uint64_t launch_count();
+// cudaFuncAttributeMaxDynamicSharedMemorySize (and, with threads > 0, the
+// max carveout + occupancy query) once per (device, kernel).
+msp_status set_smem_attr(const void *func, int smem_bytes, const char *where, int threads = 0, int *occ = nullptr);
 
 inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
@@ -70,16 +73,17 @@ size_t spgemm_setup_ws_bytes(const msp_csr *A, const msp_csr *B);
 msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_t b1, msp_spgemm_info *info,
                             cudaStream_t s);
 msp_status spgemm_symbolic_run(const msp_csr *A, const msp_csr *B, const void *ws1, size_t b1, void *ws2,
-                               size_t b2, int32_t *Crp, int64_t *nnzC, cudaStream_t s);
+                               size_t b2, msp_spgemm_info *info, int32_t *Crp, int64_t *nnzC, cudaStream_t s);
 msp_status spgemm_numeric_run(const msp_csr *A, const msp_csr *B, const void *ws1, size_t b1, void *ws2,
-                              size_t b2, const int32_t *Crp, int32_t *Ccol, void *Cval, cudaStream_t s);
+                              size_t b2, const msp_spgemm_info *info, const int32_t *Crp, int32_t *Ccol, void *Cval,
+                              cudaStream_t s);
 
 msp_status csr_check_run(const msp_csr *A, int sorted_unique, int32_t *flags_host, void *ws, size_t ws_bytes,
                          cudaStream_t s);
 size_t set_op_ws_bytes(int64_t na, int64_t nb);
 msp_status set_op_run(int op, const void *A, const void *Av, int64_t na, const void *B, const void *Bv, int64_t nb,
-                      int key_bytes, int val_bytes, void *C, void *Cv, int64_t *nC_host, void *ws, size_t ws_bytes,
-                      cudaStream_t s);
+                      int key_bytes, int val_bytes, void *C, void *Cv, int64_t cap, int64_t *nC_host, void *ws,
+                      size_t ws_bytes, cudaStream_t s);
 msp_status rebase_run(const int32_t *in, int32_t *out, int64_t n, int64_t base, cudaStream_t s);
 
 }  // namespace msp

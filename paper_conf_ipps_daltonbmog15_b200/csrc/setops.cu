@@ -175,7 +175,7 @@ __global__ void __launch_bounds__(SET_NT, MSP_SET_MINB)
 set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t na, const KT *__restrict__ B,
                 const void *__restrict__ Bv, int64_t nb, const Cut *__restrict__ cuts, int64_t ntiles,
                 uint64_t *__restrict__ states, unsigned *__restrict__ ticket, KT *__restrict__ C,
-                void *__restrict__ Cv, int64_t *__restrict__ nC)
+                void *__restrict__ Cv, int64_t cap, int64_t *__restrict__ nC, unsigned *__restrict__ bad)
 {
     using VT = typename ValT<VB>::T;
     constexpr bool EA = (OP == 0 || OP == 2 || OP == 3), EB = (OP == 0 || OP == 3), EM = (OP == 0 || OP == 1);
@@ -190,7 +190,14 @@ set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t n
     const int tile = S.tile;
 #endif
     const Cut c0 = cuts[tile], c1 = cuts[tile + 1];
-    const int la = int(c1.i - c0.i), lb = int(c1.j - c0.j);
+    // Unsorted input (a contract violation) can give non-monotone or oversized
+    // cuts: flag it (the call returns MSP_ERR_INPUT) and clamp the windows so
+    // every shared-memory and global access stays in bounds.
+    const int64_t la64 = c1.i - c0.i, lb64 = c1.j - c0.j;
+    const bool bad_cut = la64 < 0 || lb64 < 0 || la64 + lb64 > SET_T + 1;
+    const int la = int(la64 < 0 ? 0 : la64 > SET_T + 1 ? SET_T + 1 : la64);
+    const int lb = int(lb64 < 0 ? 0 : lb64 > SET_T + 1 ? SET_T + 1 : lb64);
+    if (tid == 0 && bad_cut) atomicOr(bad, 1u);
     // stage both windows with asynchronous element copies (LDGSTS): every
     // copy of the tile is in flight at once, no register round trip
     for (int x = tid; x < la; x += SET_NT) {
@@ -203,6 +210,15 @@ set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t n
     }
     cp_async_wait_all();
     __syncthreads();
+    {  // contract check: keys ascending inside the windows and across the
+       // window edges (with monotone cuts the windows tile A and B exactly)
+        bool uns = false;
+        for (int x = tid; x + 1 < la; x += SET_NT) uns |= S.ka[x + 1] < S.ka[x];
+        for (int x = tid; x + 1 < lb; x += SET_NT) uns |= S.kb[x + 1] < S.kb[x];
+        if (tid == 0 && la > 0 && c0.i > 0 && c0.i < na) uns |= S.ka[0] < A[c0.i - 1];
+        if (tid == 1 && lb > 0 && c0.j > 0 && c0.j < nb) uns |= S.kb[0] < B[c0.j - 1];
+        if (uns) atomicOr(bad, 1u);
+    }
     {  // this thread's cut inside the tile (windows clipped to the tile: consistent, R4)
         const int d = min(tid * SET_IPT, la + lb);
         const Cut c = balanced_cut<KT, int>([&](int x) { return S.ka[x]; }, la, [&](int x) { return S.kb[x]; }, lb, d);
@@ -285,7 +301,7 @@ set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t n
             int p = off;
 #pragma unroll
             for (int s = 0; s < SET_STEPS; ++s) {
-                if (emitted & (1u << s)) {
+                if ((emitted & (1u << s)) && p < SET_T + 2) {  // bound only binds on unsorted input
                     S.ka[p] = rk[s];
                     if constexpr (VB > 0) S.va[p] = rv[s];
                     ++p;
@@ -336,15 +352,18 @@ set_tile_kernel(const KT *__restrict__ A, const void *__restrict__ Av, int64_t n
     __syncthreads();
     const int64_t base = S.base;
     if (regs) {  // coalesced store of the staged run
-        for (int x = tid; x < tot; x += SET_NT) {
+        const int nst = min(tot, SET_T + 2);
+        for (int x = tid; x < nst && base + x < cap; x += SET_NT) {
             C[base + x] = S.ka[x];
             if constexpr (VB > 0) static_cast<VT *>(Cv)[base + x] = S.va[x];
         }
     } else {
         int64_t pos = base + off;
         walk([&](bool fromA, int x) {
-            C[pos] = fromA ? S.ka[x] : S.kb[x];
-            if constexpr (VB > 0) static_cast<VT *>(Cv)[pos] = fromA ? S.va[x] : S.vb[x];
+            if (pos < cap) {
+                C[pos] = fromA ? S.ka[x] : S.kb[x];
+                if constexpr (VB > 0) static_cast<VT *>(Cv)[pos] = fromA ? S.va[x] : S.vb[x];
+            }
             ++pos;
         });
     }
@@ -354,7 +373,7 @@ struct SetWs {
     Cut *cuts;
     uint64_t *states;
     unsigned *ticket;
-    int64_t *nC;
+    int64_t *nC;  // nC[0] result size, nC[1] contract-violation flag
     int64_t ntiles;
     size_t bytes;
 };
@@ -366,7 +385,7 @@ SetWs carve(int64_t na, int64_t nb, void *ws, size_t bytes, bool *ok)
     w.ntiles = items > 0 ? ceil_div(items, SET_T) : 0;
     Carve cv(ws, bytes);
     w.ticket = cv.take<unsigned>(4);
-    w.nC = cv.take<int64_t>(1);
+    w.nC = cv.take<int64_t>(2);
     w.states = cv.take<uint64_t>(size_t(w.ntiles > 0 ? w.ntiles : 1));
     w.cuts = cv.take<Cut>(size_t(w.ntiles + 1));
     w.bytes = cv.off;
@@ -376,42 +395,37 @@ SetWs carve(int64_t na, int64_t nb, void *ws, size_t bytes, bool *ok)
 
 template <typename KT, int VB, int OP>
 msp_status launch_tiles(const void *A, const void *Av, int64_t na, const void *B, const void *Bv, int64_t nb,
-                        const SetWs &w, void *C, void *Cv, cudaStream_t s)
+                        const SetWs &w, void *C, void *Cv, int64_t cap, cudaStream_t s)
 {
     auto kern = set_tile_kernel<KT, VB, OP>;
     const int smem = int(sizeof(SetSmem<KT, VB>));
-    static int configured = 0;
-    if (!configured) {
-        msp_status st = cuda_check(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem),
-                                   "set op: smem");
-        if (st != MSP_OK) return st;
-        configured = 1;
-    }
+    msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), smem, "set op: smem");
+    if (st != MSP_OK) return st;
     kern<<<unsigned(w.ntiles), SET_NT, smem, s>>>(static_cast<const KT *>(A), Av, na, static_cast<const KT *>(B), Bv,
                                                   nb, w.cuts, w.ntiles, w.states, w.ticket, static_cast<KT *>(C), Cv,
-                                                  w.nC);
+                                                  cap, w.nC, reinterpret_cast<unsigned *>(w.nC + 1));
     return last_launch("set_tile_kernel");
 }
 
 template <typename KT, int VB>
 msp_status launch_op(int op, const void *A, const void *Av, int64_t na, const void *B, const void *Bv, int64_t nb,
-                     const SetWs &w, void *C, void *Cv, cudaStream_t s)
+                     const SetWs &w, void *C, void *Cv, int64_t cap, cudaStream_t s)
 {
     switch (op) {
-    case 0: return launch_tiles<KT, VB, 0>(A, Av, na, B, Bv, nb, w, C, Cv, s);
-    case 1: return launch_tiles<KT, VB, 1>(A, Av, na, B, Bv, nb, w, C, Cv, s);
-    case 2: return launch_tiles<KT, VB, 2>(A, Av, na, B, Bv, nb, w, C, Cv, s);
-    default: return launch_tiles<KT, VB, 3>(A, Av, na, B, Bv, nb, w, C, Cv, s);
+    case 0: return launch_tiles<KT, VB, 0>(A, Av, na, B, Bv, nb, w, C, Cv, cap, s);
+    case 1: return launch_tiles<KT, VB, 1>(A, Av, na, B, Bv, nb, w, C, Cv, cap, s);
+    case 2: return launch_tiles<KT, VB, 2>(A, Av, na, B, Bv, nb, w, C, Cv, cap, s);
+    default: return launch_tiles<KT, VB, 3>(A, Av, na, B, Bv, nb, w, C, Cv, cap, s);
     }
 }
 
 template <typename KT>
 msp_status launch_kv(int op, int vb, const void *A, const void *Av, int64_t na, const void *B, const void *Bv,
-                     int64_t nb, const SetWs &w, void *C, void *Cv, cudaStream_t s)
+                     int64_t nb, const SetWs &w, void *C, void *Cv, int64_t cap, cudaStream_t s)
 {
-    if (vb == 0) return launch_op<KT, 0>(op, A, Av, na, B, Bv, nb, w, C, Cv, s);
-    if (vb == 4) return launch_op<KT, 4>(op, A, Av, na, B, Bv, nb, w, C, Cv, s);
-    return launch_op<KT, 8>(op, A, Av, na, B, Bv, nb, w, C, Cv, s);
+    if (vb == 0) return launch_op<KT, 0>(op, A, Av, na, B, Bv, nb, w, C, Cv, cap, s);
+    if (vb == 4) return launch_op<KT, 4>(op, A, Av, na, B, Bv, nb, w, C, Cv, cap, s);
+    return launch_op<KT, 8>(op, A, Av, na, B, Bv, nb, w, C, Cv, cap, s);
 }
 
 }  // namespace
@@ -423,8 +437,8 @@ size_t set_op_ws_bytes(int64_t na, int64_t nb)
 }
 
 msp_status set_op_run(int op, const void *A, const void *Av, int64_t na, const void *B, const void *Bv, int64_t nb,
-                      int key_bytes, int val_bytes, void *C, void *Cv, int64_t *nC_host, void *ws, size_t ws_bytes,
-                      cudaStream_t s)
+                      int key_bytes, int val_bytes, void *C, void *Cv, int64_t cap, int64_t *nC_host, void *ws,
+                      size_t ws_bytes, cudaStream_t s)
 {
     bool ok;
     SetWs w = carve(na, nb, ws, ws_bytes, &ok);
@@ -447,24 +461,28 @@ msp_status set_op_run(int op, const void *A, const void *Av, int64_t na, const v
         st = last_launch("set_partition_kernel");
         if (st != MSP_OK) return st;
     }
-    st = (key_bytes == 4) ? launch_kv<uint32_t>(op, val_bytes, A, Av, na, B, Bv, nb, w, C, Cv, s)
-                          : launch_kv<uint64_t>(op, val_bytes, A, Av, na, B, Bv, nb, w, C, Cv, s);
+    st = (key_bytes == 4) ? launch_kv<uint32_t>(op, val_bytes, A, Av, na, B, Bv, nb, w, C, Cv, cap, s)
+                          : launch_kv<uint64_t>(op, val_bytes, A, Av, na, B, Bv, nb, w, C, Cv, cap, s);
     if (st != MSP_OK) return st;
     // the result size comes back through a pinned word (a pageable
     // destination would stage the 8-byte copy through a driver buffer)
     static thread_local int64_t *pinned = nullptr;
     if (!pinned) {
-        st = cuda_check(cudaMallocHost(reinterpret_cast<void **>(&pinned), sizeof(int64_t)), "set op: pinned size");
+        st = cuda_check(cudaMallocHost(reinterpret_cast<void **>(&pinned), 2 * sizeof(int64_t)), "set op: pinned size");
         if (st != MSP_OK) {
             pinned = nullptr;
             return st;
         }
     }
-    st = cuda_check(cudaMemcpyAsync(pinned, w.nC, sizeof(int64_t), cudaMemcpyDeviceToHost, s), "set op: size");
+    st = cuda_check(cudaMemcpyAsync(pinned, w.nC, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, s), "set op: size");
     if (st != MSP_OK) return st;
     st = cuda_check(cudaStreamSynchronize(s), "set op: sync");
     if (st != MSP_OK) return st;
-    *nC_host = *pinned;
+    *nC_host = pinned[0];
+    if (pinned[1]) {
+        set_error("set op: keys are not sorted ascending (as unsigned %d-byte integers)", key_bytes);
+        return MSP_ERR_INPUT;
+    }
     return MSP_OK;
 }
 

@@ -426,13 +426,8 @@ msp_status launch_tiles(const msp_csr *A, const msp_csr *B, const AddWs &w, int3
 {
     auto kern = spadd_tile_kernel<V, FILL>;
     const int smem = AddLayout<V, FILL>::BYTES;
-    static int configured = 0;
-    if (!configured) {
-        msp_status st = cuda_check(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem),
-                                   "spadd: smem");
-        if (st != MSP_OK) return st;
-        configured = 1;
-    }
+    msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), smem, "spadd: smem");
+    if (st != MSP_OK) return st;
     kern<<<unsigned(w.ntiles), ADD_NT, smem, s>>>(
         A->nrows, A->row_offsets, A->col_idx, static_cast<const V *>(A->vals), B->row_offsets, B->col_idx,
         static_cast<const V *>(B->vals), A->nnz, B->nnz, w.splits, w.tile_count, w.tile_off, Crp ? Crp + 1 : nullptr, Ccol,

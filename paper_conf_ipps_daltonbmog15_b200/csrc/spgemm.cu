@@ -121,7 +121,7 @@ struct SetupWs {
     int64_t *longO;      // [m + 1] prefix of longP
     int64_t *longC;      // [m]  chunks of the i-th long row
     int64_t *longCO;     // [m + 1] prefix of longC
-    unsigned long long *stats;  // [4]: max row products
+    unsigned long long *stats;  // [8]: [0] max row products, [1..5] gathered setup sizes
     void *scan;
     size_t scan_bytes;
     size_t bytes;
@@ -142,7 +142,7 @@ SetupWs carve_setup(const msp_csr *A, void *ws, size_t cap, bool *ok)
     w.longO = cv.take<int64_t>(size_t(m + 1));
     w.longC = cv.take<int64_t>(size_t(m > 0 ? m : 1));
     w.longCO = cv.take<int64_t>(size_t(m + 1));
-    w.stats = cv.take<unsigned long long>(4);
+    w.stats = cv.take<unsigned long long>(8);
     w.scan_bytes = scan_ws_bytes(std::max<int64_t>(std::max<int64_t>(m, nnz), 1));
     w.scan = cv.take<char>(w.scan_bytes);
     w.bytes = cv.off;
@@ -785,29 +785,58 @@ MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, void *ws, size_t cap, b
     return w;
 }
 
-struct HostInfo {  // read back by setup, re-derived by symbolic / numeric
+struct HostInfo {  // read back by setup (one synchronisation), passed to symbolic / numeric in msp_spgemm_info
     int64_t nprods, nlong, LP, LC, maxP;
 };
 
+// The setup sizes gathered into one device array (so setup reads them back
+// with ONE copy and one synchronisation): S[nnzA], longpos[m], longO[nlong],
+// longCO[nlong], max row products.
+__global__ void info_gather_kernel(const int64_t *__restrict__ S, int64_t nnzA, const int64_t *__restrict__ longpos,
+                                   int64_t m, const int64_t *__restrict__ longO, const int64_t *__restrict__ longCO,
+                                   const unsigned long long *__restrict__ stats, int64_t *__restrict__ out)
+{
+    if (threadIdx.x != 0) return;
+    const int64_t nlong = longpos[m];
+    out[0] = S[nnzA];
+    out[1] = nlong;
+    out[2] = nlong > 0 ? longO[nlong] : 0;
+    out[3] = nlong > 0 ? longCO[nlong] : 0;
+    out[4] = int64_t(stats[0]);
+}
+
+// A pinned host staging word array per host thread for the synchronising reads.
+int64_t *pinned_words()
+{
+    static thread_local int64_t *p = nullptr;
+    if (!p && cudaMallocHost(reinterpret_cast<void **>(&p), 8 * sizeof(int64_t)) != cudaSuccess) p = nullptr;
+    return p;
+}
+
+msp_status read_back(const int64_t *dev, int n, int64_t *host, cudaStream_t s, const char *where)
+{
+    int64_t *pin = pinned_words();
+    msp_status st = cuda_check(cudaMemcpyAsync(pin ? pin : host, dev, size_t(n) * 8, cudaMemcpyDeviceToHost, s), where);
+    if (st == MSP_OK) st = cuda_check(cudaStreamSynchronize(s), where);
+    if (st == MSP_OK && pin)
+        for (int i = 0; i < n; ++i) host[i] = pin[i];
+    return st;
+}
+
 msp_status read_info(const SetupWs &sw, int64_t m, int64_t nnzA, HostInfo *h, cudaStream_t s)
 {
-    int64_t v[5] = {0, 0, 0, 0, 0};
-    msp_status st = cuda_check(cudaMemcpyAsync(&v[0], &sw.S[nnzA], 8, cudaMemcpyDeviceToHost, s), "spgemm: info");
-    if (st == MSP_OK) st = cuda_check(cudaMemcpyAsync(&v[1], &sw.longpos[m], 8, cudaMemcpyDeviceToHost, s), "info");
-    if (st == MSP_OK) st = cuda_check(cudaMemcpyAsync(&v[4], sw.stats, 8, cudaMemcpyDeviceToHost, s), "info");
-    if (st == MSP_OK) st = cuda_check(cudaStreamSynchronize(s), "spgemm: sync");
+    info_gather_kernel<<<1, 32, 0, s>>>(sw.S, nnzA, sw.longpos, m, sw.longO, sw.longCO, sw.stats,
+                                        reinterpret_cast<int64_t *>(sw.stats) + 1);
+    msp_status st = last_launch("info_gather_kernel");
+    if (st != MSP_OK) return st;
+    int64_t v[5];
+    st = read_back(reinterpret_cast<const int64_t *>(sw.stats) + 1, 5, v, s, "spgemm: setup sizes");
     if (st != MSP_OK) return st;
     h->nprods = v[0];
     h->nlong = v[1];
-    h->maxP = v[4];
-    if (h->nlong > 0) {
-        st = cuda_check(cudaMemcpyAsync(&v[2], &sw.longO[h->nlong], 8, cudaMemcpyDeviceToHost, s), "info");
-        if (st == MSP_OK) st = cuda_check(cudaMemcpyAsync(&v[3], &sw.longCO[h->nlong], 8, cudaMemcpyDeviceToHost, s), "info");
-        if (st == MSP_OK) st = cuda_check(cudaStreamSynchronize(s), "spgemm: sync");
-        if (st != MSP_OK) return st;
-    }
     h->LP = v[2];
     h->LC = v[3];
+    h->maxP = v[4];
     return MSP_OK;
 }
 
@@ -817,13 +846,8 @@ msp_status launch_tiles(const msp_csr *A, const msp_csr *B, const SetupWs &sw, c
 {
     auto kern = gemm_tile_kernel<KT, V, NUM>;
     const int smem = int(sizeof(TileSmem<KT, NUM>));
-    static int configured = 0;
-    if (!configured) {
-        msp_status st = cuda_check(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem),
-                                   "spgemm: tile smem");
-        if (st != MSP_OK) return st;
-        configured = 1;
-    }
+    msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), smem, "spgemm: tile smem");
+    if (st != MSP_OK) return st;
     kern<<<unsigned(ntiles), GM_NT, smem, s>>>(A->col_idx, static_cast<const V *>(A->vals), B->row_offsets,
                                                 B->col_idx, static_cast<const V *>(B->vals), sw.arow, sw.S,
                                                 sw.rowlong, mw.splits, cbits, mw.perm, Crp, Ccol,
@@ -852,17 +876,12 @@ msp_status run_long(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const
     if (h.nlong == 0 || h.LP == 0) return MSP_OK;
     auto ck = long_chunk_kernel<V, NUM>;
     const int smem = int(sizeof(LongSmem<V, NUM>));
-    static int configured = 0;
-    if (!configured) {
-        msp_status st = cuda_check(cudaFuncSetAttribute(ck, cudaFuncAttributeMaxDynamicSharedMemorySize, smem),
-                                   "spgemm: chunk smem");
-        if (st != MSP_OK) return st;
-        configured = 1;
-    }
+    msp_status st = set_smem_attr(reinterpret_cast<const void *>(ck), smem, "spgemm: chunk smem");
+    if (st != MSP_OK) return st;
     ck<<<unsigned(h.LC), GM_NT, smem, s>>>(A->row_offsets, A->col_idx, static_cast<const V *>(A->vals),
                                            B->row_offsets, B->col_idx, static_cast<const V *>(B->vals), sw.S,
                                            h.nlong, sw.longrow, sw.longP, sw.longO, sw.longCO, mw.Xc[0], mw.Xv[0]);
-    msp_status st = last_launch("long_chunk_kernel");
+    st = last_launch("long_chunk_kernel");
     if (st != MSP_OK) return st;
     int cur = 0;
     int64_t maxlong = h.maxP;
@@ -892,16 +911,25 @@ msp_status run_long(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const
 int64_t ntiles_of(int64_t nnzA, int64_t nprods) { return ceil_div(nnzA + nprods > 0 ? nnzA + nprods : 1, GM_TP); }
 
 msp_status prepare_main(const msp_csr *A, const void *ws1, size_t b1, void *ws2, size_t b2, SetupWs *sw, MainWs *mw,
-                        HostInfo *h, cudaStream_t s)
+                        const HostInfo &h)
 {
     bool ok1, ok2;
     *sw = carve_setup(A, const_cast<void *>(ws1), b1, &ok1);
     if (!ok1) return MSP_ERR_WORKSPACE;
-    msp_status st = read_info(*sw, A->nrows, A->nnz, h, s);
-    if (st != MSP_OK) return st;
-    *mw = carve_main(A->nrows, ntiles_of(A->nnz, h->nprods), h->LP, ws2, b2, &ok2);
+    *mw = carve_main(A->nrows, ntiles_of(A->nnz, h.nprods), h.LP, ws2, b2, &ok2);
     if (!ok2) return MSP_ERR_WORKSPACE;
     return MSP_OK;
+}
+
+HostInfo host_info(const msp_spgemm_info *info)
+{
+    HostInfo h;
+    h.nprods = info->nprods;
+    h.nlong = info->long_rows;
+    h.LP = info->long_products;
+    h.LC = info->long_chunks;
+    h.maxP = info->max_row_products;
+    return h;
 }
 
 }  // namespace
@@ -920,7 +948,7 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
     SetupWs w = carve_setup(A, ws1, b1, &ok);
     if (!ok) return MSP_ERR_WORKSPACE;
     const int64_t m = A->nrows, nnz = A->nnz;
-    msp_status st = cuda_check(cudaMemsetAsync(w.stats, 0, 4 * sizeof(unsigned long long), s), "spgemm: clear");
+    msp_status st = cuda_check(cudaMemsetAsync(w.stats, 0, 8 * sizeof(unsigned long long), s), "spgemm: clear");
     if (st != MSP_OK) return st;
     if (nnz > 0) {
         const int64_t thr = ceil_div(m + nnz, AROW_ITEMS);
@@ -964,25 +992,34 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
     info->long_products = h.LP;
     info->max_row_products = h.maxP;
     info->main_ws_bytes = int64_t(mw.bytes + 256);
+    info->long_chunks = h.LC;
+    info->max_tile_span = -1;  // set by symbolic
     return MSP_OK;
 }
 
+// Symbolic: partition, tile spans (ONE synchronisation: the key width of the
+// tile launch depends on the largest tile row span), tile + long-row passes,
+// scan of the row counts (second synchronisation: nnz(C)).  Numeric: the same
+// launches with values, every size taken from the host info -- no
+// synchronisation.
 template <bool NUM>
 msp_status spgemm_pass(const msp_csr *A, const msp_csr *B, const void *ws1, size_t b1, void *ws2, size_t b2,
-                       int32_t *Crp, int32_t *Ccol, void *Cval, int64_t *nnzC, cudaStream_t s)
+                       msp_spgemm_info *info, int32_t *Crp, int32_t *Ccol, void *Cval, int64_t *nnzC, cudaStream_t s)
 {
     SetupWs sw;
     MainWs mw;
-    HostInfo h;
-    msp_status st = prepare_main(A, ws1, b1, ws2, b2, &sw, &mw, &h, s);
+    const HostInfo h = host_info(info);
+    msp_status st = prepare_main(A, ws1, b1, ws2, b2, &sw, &mw, h);
     if (st != MSP_OK) return st;
     const int64_t m = A->nrows;
     const int64_t ntiles = ntiles_of(A->nnz, h.nprods);
+    int64_t maxspan = info->max_tile_span;
     if (!NUM) {
         st = cuda_check(cudaMemsetAsync(Crp, 0, size_t(m + 1) * sizeof(int32_t), s), "spgemm: clear rp");
         if (st != MSP_OK) return st;
         if (m == 0) {
             *nnzC = 0;
+            info->max_tile_span = 0;
             return cuda_check(cudaStreamSynchronize(s), "spgemm: sync");
         }
         gemm_partition_kernel<<<unsigned(std::min<int64_t>(ceil_div(ntiles + 1, 256), 148 * 16)), 256, 0, s>>>(
@@ -995,13 +1032,15 @@ msp_status spgemm_pass(const msp_csr *A, const msp_csr *B, const void *ws1, size
             ntiles, mw.splits, sw.arow, reinterpret_cast<unsigned long long *>(&mw.totals[1]));
         st = last_launch("tile_span_kernel");
         if (st != MSP_OK) return st;
+        st = read_back(&mw.totals[1], 1, &maxspan, s, "spgemm: tile span");
+        if (st != MSP_OK) return st;
+        info->max_tile_span = maxspan;
     } else if (m == 0 || h.nprods == 0) {
         return MSP_OK;
+    } else if (maxspan < 0) {
+        set_error("spgemm: numeric needs the info returned by symbolic (max_tile_span unset)");
+        return MSP_ERR_ARG;
     }
-    int64_t maxspan = 0;  // written by the symbolic pass, kept in main_ws for numeric
-    st = cuda_check(cudaMemcpyAsync(&maxspan, &mw.totals[1], 8, cudaMemcpyDeviceToHost, s), "spgemm: span");
-    if (st == MSP_OK) st = cuda_check(cudaStreamSynchronize(s), "spgemm: sync");
-    if (st != MSP_OK) return st;
     if (h.nprods > 0) {
         st = (A->dtype == MSP_F64) ? run_tiles<double, NUM>(A, B, sw, mw, ntiles, maxspan, Crp, Ccol, Cval, s)
                                    : run_tiles<float, NUM>(A, B, sw, mw, ntiles, maxspan, Crp, Ccol, Cval, s);
@@ -1014,8 +1053,7 @@ msp_status spgemm_pass(const msp_csr *A, const msp_csr *B, const void *ws1, size
         st = scan_counts_to_offsets_i32(Crp + 1, m, &mw.totals[0], mw.scan, mw.scan_bytes, s);
         if (st != MSP_OK) return st;
         int64_t tot = 0;
-        st = cuda_check(cudaMemcpyAsync(&tot, &mw.totals[0], 8, cudaMemcpyDeviceToHost, s), "spgemm: nnz");
-        if (st == MSP_OK) st = cuda_check(cudaStreamSynchronize(s), "spgemm: sync");
+        st = read_back(&mw.totals[0], 1, &tot, s, "spgemm: nnz");
         if (st != MSP_OK) return st;
         *nnzC = tot;
         if (tot > INT32_MAX) {
@@ -1027,15 +1065,17 @@ msp_status spgemm_pass(const msp_csr *A, const msp_csr *B, const void *ws1, size
 }
 
 msp_status spgemm_symbolic_run(const msp_csr *A, const msp_csr *B, const void *ws1, size_t b1, void *ws2,
-                               size_t b2, int32_t *Crp, int64_t *nnzC, cudaStream_t s)
+                               size_t b2, msp_spgemm_info *info, int32_t *Crp, int64_t *nnzC, cudaStream_t s)
 {
-    return spgemm_pass<false>(A, B, ws1, b1, ws2, b2, Crp, nullptr, nullptr, nnzC, s);
+    return spgemm_pass<false>(A, B, ws1, b1, ws2, b2, info, Crp, nullptr, nullptr, nnzC, s);
 }
 
 msp_status spgemm_numeric_run(const msp_csr *A, const msp_csr *B, const void *ws1, size_t b1, void *ws2,
-                              size_t b2, const int32_t *Crp, int32_t *Ccol, void *Cval, cudaStream_t s)
+                              size_t b2, const msp_spgemm_info *info, const int32_t *Crp, int32_t *Ccol, void *Cval,
+                              cudaStream_t s)
 {
-    return spgemm_pass<true>(A, B, ws1, b1, ws2, b2, const_cast<int32_t *>(Crp), Ccol, Cval, nullptr, s);
+    msp_spgemm_info copy = *info;
+    return spgemm_pass<true>(A, B, ws1, b1, ws2, b2, &copy, const_cast<int32_t *>(Crp), Ccol, Cval, nullptr, s);
 }
 
 }  // namespace msp

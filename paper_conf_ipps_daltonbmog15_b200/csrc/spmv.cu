@@ -714,25 +714,10 @@ template <typename V, class C>
 msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
 {
     auto kern = spmv_merge_kernel<V, C>;
-    static int configured = 0;
-    static int occ = 1;
-    if (!configured) {
-        msp_status st = cuda_check(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM),
-                                   "spmv: set smem");
-        if (st != MSP_OK) return st;
-        st = cuda_check(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100),
-                        "spmv: carveout");
-        if (st != MSP_OK) return st;
-        st = cuda_check(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, C::THREADS, C::SMEM),
-                        "spmv: occupancy");
-        if (getenv("MSP_VERBOSE"))
-            fprintf(stderr, "msp spmv: rowk=%d K=%d NW=%d T=%d stages=%d smem=%d occupancy=%d CTAs/SM\n", int(C::ROWK), C::K,
-                    C::NW, C::T, C::STAGES, C::SMEM, occ);
-        if (st != MSP_OK) return st;
-        if (occ < 1) occ = 1;
-        if (occ > 4) occ = 4;
-        configured = 1;
-    }
+    int occ = 1;
+    msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), C::SMEM, "spmv: smem", C::THREADS, &occ);
+    if (st != MSP_OK) return st;
+    if (occ > 4) occ = 4;
     if (A->nrows == 0) return MSP_OK;
     if (A->nnz == 0)  // every row is empty: y = +0.0 (Z6)
         return cuda_check(cudaMemsetAsync(y, 0, size_t(A->nrows) * sizeof(V), s), "spmv: zero y");

@@ -9,6 +9,7 @@ spgemm (III-C).
 from __future__ import annotations
 
 import ctypes
+import itertools
 from dataclasses import dataclass
 
 import torch
@@ -61,20 +62,38 @@ class CsrTensor:
 # ----------------------------------------------------------------- workspaces
 
 _WS: dict = {}
+_OWNER: dict = {}
+_TOKENS = itertools.count(1)
+
+
+def _ws_key(device, slot: str, stream=None):
+    dev = torch.device(device)
+    s = stream if stream is not None else torch.cuda.current_stream(dev)
+    return (dev.index, s.cuda_stream, slot)
 
 
 def workspace(nbytes: int, device, slot: str, stream=None) -> torch.Tensor:
     """Zero-initialised byte workspace cached per (device, stream, slot).  Each
     slot is only ever used by one kind of call, whose kernels leave their
-    counters zeroed, so reuse needs no re-clearing."""
-    dev = torch.device(device)
-    s = stream if stream is not None else torch.cuda.current_stream(dev)
-    key = (dev.index, s.cuda_stream, slot)
+    counters zeroed, so reuse needs no re-clearing.  Symbolic -> numeric
+    state kept in a slot belongs to the plan that last ran its symbolic
+    phase there (see _claim / _owns)."""
+    key = _ws_key(device, slot, stream)
     buf = _WS.get(key)
     if buf is None or buf.numel() < nbytes:
-        buf = torch.zeros(max(int(nbytes), 256), dtype=torch.uint8, device=dev)
+        buf = torch.zeros(max(int(nbytes), 256), dtype=torch.uint8, device=torch.device(device))
         _WS[key] = buf
+        _OWNER.pop(key, None)
     return buf
+
+
+def _claim(token: int, device, slots, stream=None) -> None:
+    for sl in slots:
+        _OWNER[_ws_key(device, sl, stream)] = token
+
+
+def _owns(token: int, device, slots, stream=None) -> bool:
+    return all(_OWNER.get(_ws_key(device, sl, stream)) == token for sl in slots)
 
 
 def _stream_ptr(device, stream=None):
@@ -117,21 +136,27 @@ class SpAddPlan:
         n = ctypes.c_size_t(0)
         check("msp_spadd_workspace", lib().msp_spadd_workspace(ctypes.byref(self.a), ctypes.byref(self.b),
                                                                ctypes.byref(n)))
-        self.ws = workspace(int(n.value), A.device, "spadd", stream)
+        self.ws_bytes = int(n.value)
+        self.ws = workspace(self.ws_bytes, A.device, "spadd", stream)
         self.rp = torch.empty(A.shape[0] + 1, dtype=torch.int32, device=A.device)
         self.nnz = None
+        self.token = next(_TOKENS)
 
     def symbolic(self) -> int:
         nnz = ctypes.c_int64(0)
+        self.ws = workspace(self.ws_bytes, self.A.device, "spadd", self.stream)
         check("msp_spadd_symbolic",
               lib().msp_spadd_symbolic(ctypes.byref(self.a), ctypes.byref(self.b), self.rp.data_ptr(),
                                        ctypes.byref(nnz), self.ws.data_ptr(), self.ws.numel(),
                                        _stream_ptr(self.A.device, self.stream)))
+        _claim(self.token, self.A.device, ("spadd",), self.stream)
         self.nnz = int(nnz.value)
         return self.nnz
 
     def numeric(self, col: torch.Tensor | None = None, val: torch.Tensor | None = None) -> CsrTensor:
-        if self.nnz is None:
+        # numeric needs the partition this plan's symbolic call left in the
+        # shared workspace; if another plan has used it since, redo symbolic
+        if self.nnz is None or not _owns(self.token, self.A.device, ("spadd",), self.stream):
             self.symbolic()
         dev = self.A.device
         col = col if col is not None else torch.empty(self.nnz, dtype=torch.int32, device=dev)
@@ -164,19 +189,26 @@ class SpGemmPlan:
         n = ctypes.c_size_t(0)
         check("msp_spgemm_setup_workspace",
               lib().msp_spgemm_setup_workspace(ctypes.byref(self.a), ctypes.byref(self.b), ctypes.byref(n)))
-        self.ws1 = workspace(int(n.value), A.device, "spgemm_setup", stream)
+        self.ws1_bytes = int(n.value)
+        self.ws1 = workspace(self.ws1_bytes, A.device, "spgemm_setup", stream)
         self.info = None
         self.ws2 = None
         self.rp = torch.empty(A.shape[0] + 1, dtype=torch.int32, device=A.device)
         self.nnz = None
+        self.token = next(_TOKENS)
+
+    _SLOTS = ("spgemm_setup", "spgemm_main")
 
     def setup(self) -> msp_spgemm_info:
         info = msp_spgemm_info()
+        self.ws1 = workspace(self.ws1_bytes, self.A.device, "spgemm_setup", self.stream)
         check("msp_spgemm_setup",
               lib().msp_spgemm_setup(ctypes.byref(self.a), ctypes.byref(self.b), self.ws1.data_ptr(),
                                      self.ws1.numel(), ctypes.byref(info), _stream_ptr(self.A.device, self.stream)))
         self.info = info
         self.ws2 = workspace(int(info.main_ws_bytes), self.A.device, "spgemm_main", self.stream)
+        _claim(self.token, self.A.device, self._SLOTS[:1], self.stream)
+        self.nnz = None  # symbolic must follow a setup
         return info
 
     @property
@@ -186,25 +218,31 @@ class SpGemmPlan:
         return int(self.info.nprods)
 
     def symbolic(self) -> int:
-        if self.info is None:
+        if self.info is None or not _owns(self.token, self.A.device, self._SLOTS[:1], self.stream):
             self.setup()
         nnz = ctypes.c_int64(0)
         check("msp_spgemm_symbolic",
               lib().msp_spgemm_symbolic(ctypes.byref(self.a), ctypes.byref(self.b), self.ws1.data_ptr(),
-                                        self.ws1.numel(), self.ws2.data_ptr(), self.ws2.numel(), self.rp.data_ptr(),
-                                        ctypes.byref(nnz), _stream_ptr(self.A.device, self.stream)))
+                                        self.ws1.numel(), self.ws2.data_ptr(), self.ws2.numel(),
+                                        ctypes.byref(self.info), self.rp.data_ptr(), ctypes.byref(nnz),
+                                        _stream_ptr(self.A.device, self.stream)))
+        _claim(self.token, self.A.device, self._SLOTS, self.stream)
         self.nnz = int(nnz.value)
         return self.nnz
 
     def numeric(self, col: torch.Tensor | None = None, val: torch.Tensor | None = None) -> CsrTensor:
-        if self.nnz is None:
+        # numeric reads the setup arrays and the tile permutations this plan's
+        # symbolic call left in the shared workspaces; redo them if another
+        # plan has used those workspaces since
+        if self.nnz is None or not _owns(self.token, self.A.device, self._SLOTS, self.stream):
             self.symbolic()
         dev = self.A.device
         col = col if col is not None else torch.empty(self.nnz, dtype=torch.int32, device=dev)
         val = val if val is not None else torch.empty(self.nnz, dtype=self.A.dtype, device=dev)
         check("msp_spgemm_numeric",
               lib().msp_spgemm_numeric(ctypes.byref(self.a), ctypes.byref(self.b), self.ws1.data_ptr(),
-                                       self.ws1.numel(), self.ws2.data_ptr(), self.ws2.numel(), self.rp.data_ptr(),
+                                       self.ws1.numel(), self.ws2.data_ptr(), self.ws2.numel(),
+                                       ctypes.byref(self.info), self.rp.data_ptr(),
                                        col.data_ptr() if self.nnz else None, val.data_ptr() if self.nnz else None,
                                        _stream_ptr(dev, self.stream)))
         return CsrTensor(self.rp, col, val, (self.A.shape[0], self.B.shape[1]))
