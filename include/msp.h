@@ -27,6 +27,13 @@
  * SpMV accepts any column order.  Indices are int32; product counts (Nprods)
  * are int64 internally.
  *
+ * Debug validation: with MSP_DEBUG_VALIDATE=1 in the environment (read once
+ * per process), msp_spmv, msp_spadd_symbolic and msp_spgemm_setup first run
+ * msp_csr_check on their inputs (sorted-unique columns required for SpAdd /
+ * SpGEMM), synchronise, and return MSP_ERR_INPUT on a malformed matrix.  The
+ * check's flag word lives in the last bytes of the workspace, which is why
+ * every *_workspace size includes 512 bytes of tail room.
+ *
  * Ownership: the caller allocates and owns every device buffer (inputs,
  * outputs, workspaces).  The library never calls cudaMalloc/cudaFree and
  * keeps no pointer after a call returns, except that the workspaces named in

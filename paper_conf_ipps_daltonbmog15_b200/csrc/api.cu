@@ -4,6 +4,7 @@
 // launch; the kernels live in spmv.cu / spadd.cu / spgemm.cu / scan.cu /
 // check.cu.  No call allocates device memory: every buffer is the caller's.
 #include <cstdarg>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <atomic>
@@ -126,6 +127,35 @@ msp_status check_csr(const msp_csr *A, const char *name)
 
 inline cudaStream_t as_stream(void *s) { return static_cast<cudaStream_t>(s); }
 
+// Every *_workspace size carries kValidateBytes of tail room for the
+// MSP_DEBUG_VALIDATE input check (a flag word; the library never allocates).
+constexpr size_t kValidateBytes = 512;
+
+bool debug_validate_on()
+{
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("MSP_DEBUG_VALIDATE");
+        v = (e && *e && atoi(e) != 0) ? 1 : 0;
+    }
+    return v != 0;
+}
+
+// With MSP_DEBUG_VALIDATE=1 in the environment, the entry points run
+// msp_csr_check on their inputs first (synchronising) and return
+// MSP_ERR_INPUT on a malformed matrix instead of computing on it.
+msp_status debug_validate(const msp_csr *A, int sorted_unique, void *ws, size_t ws_bytes, size_t used, cudaStream_t s,
+                          const char *what)
+{
+    if (!debug_validate_on()) return MSP_OK;
+    const size_t off = align_up(used, 256);
+    if (off + 16 > ws_bytes) return MSP_ERR_WORKSPACE;
+    int32_t flags = 0;
+    msp_status st = csr_check_run(A, sorted_unique, &flags, static_cast<char *>(ws) + off, 16, s);
+    if (st == MSP_ERR_INPUT) set_error("%s: MSP_DEBUG_VALIDATE: malformed CSR (flags %d)", what, flags);
+    return st;
+}
+
 }  // namespace
 
 extern "C" {
@@ -160,7 +190,7 @@ msp_status msp_spmv_workspace(const msp_csr *A, size_t *bytes)
     msp_status st = check_csr(A, "A");
     if (st != MSP_OK) return st;
     if (!bytes) return MSP_ERR_ARG;
-    *bytes = spmv_ws_bytes(A);
+    *bytes = spmv_ws_bytes(A) + kValidateBytes;
     return MSP_OK;
 }
 
@@ -177,6 +207,8 @@ msp_status msp_spmv(const msp_csr *A, const void *x, void *y, void *ws, size_t w
         set_error("spmv: workspace %zu < %zu bytes", ws_bytes, spmv_ws_bytes(A));
         return MSP_ERR_WORKSPACE;
     }
+    st = debug_validate(A, 0, ws, ws_bytes, spmv_ws_bytes(A), as_stream(stream), "spmv A");
+    if (st != MSP_OK) return st;
     return spmv_run(A, x, y, ws, ws_bytes, as_stream(stream));
 }
 
@@ -203,7 +235,7 @@ msp_status msp_spadd_workspace(const msp_csr *A, const msp_csr *B, size_t *bytes
     msp_status st = check_pair_add(A, B);
     if (st != MSP_OK) return st;
     if (!bytes) return MSP_ERR_ARG;
-    *bytes = spadd_ws_bytes(A, B);
+    *bytes = spadd_ws_bytes(A, B) + kValidateBytes;
     return MSP_OK;
 }
 
@@ -215,6 +247,9 @@ msp_status msp_spadd_symbolic(const msp_csr *A, const msp_csr *B, int32_t *C_row
     if (st != MSP_OK) return st;
     if (!C_row_offsets || !nnzC_host || !ws) return MSP_ERR_ARG;
     if (ws_bytes < spadd_ws_bytes(A, B)) return MSP_ERR_WORKSPACE;
+    st = debug_validate(A, 1, ws, ws_bytes, spadd_ws_bytes(A, B), as_stream(stream), "spadd A");
+    if (st == MSP_OK) st = debug_validate(B, 1, ws, ws_bytes, spadd_ws_bytes(A, B), as_stream(stream), "spadd B");
+    if (st != MSP_OK) return st;
     return spadd_symbolic_run(A, B, C_row_offsets, nnzC_host, ws, ws_bytes, as_stream(stream));
 }
 
@@ -252,7 +287,7 @@ msp_status msp_spgemm_setup_workspace(const msp_csr *A, const msp_csr *B, size_t
     msp_status st = check_pair_mul(A, B);
     if (st != MSP_OK) return st;
     if (!bytes) return MSP_ERR_ARG;
-    *bytes = spgemm_setup_ws_bytes(A, B);
+    *bytes = spgemm_setup_ws_bytes(A, B) + kValidateBytes;
     return MSP_OK;
 }
 
@@ -264,6 +299,10 @@ msp_status msp_spgemm_setup(const msp_csr *A, const msp_csr *B, void *setup_ws, 
     if (st != MSP_OK) return st;
     if (!setup_ws || !info_host) return MSP_ERR_ARG;
     if (setup_ws_bytes < spgemm_setup_ws_bytes(A, B)) return MSP_ERR_WORKSPACE;
+    st = debug_validate(A, 1, setup_ws, setup_ws_bytes, spgemm_setup_ws_bytes(A, B), as_stream(stream), "spgemm A");
+    if (st == MSP_OK)
+        st = debug_validate(B, 1, setup_ws, setup_ws_bytes, spgemm_setup_ws_bytes(A, B), as_stream(stream), "spgemm B");
+    if (st != MSP_OK) return st;
     return spgemm_setup_run(A, B, setup_ws, setup_ws_bytes, info_host, as_stream(stream));
 }
 

@@ -63,6 +63,7 @@ struct CtaRecord {  // one per CTA in the workspace
 template <typename V, int NW_, int STAGES_, int RSLOTS_, int MINB_>
 struct Cfg {
     static constexpr bool ROWK = false;
+    static constexpr int PFW = 0;                        // x prefetch warps
     static constexpr int NW = NW_;
     static constexpr int K = 8;
     static constexpr int WSPAN = 32 * K;                 // products per worker warp
@@ -90,16 +91,17 @@ struct Cfg {
 // when rows are about K long, gather u of the 32 lanes touches the same
 // stencil position of 32 consecutive rows -- a few x cache lines per
 // instruction instead of one per row.
-template <typename V, int NW_, int K_, int STAGES_, int MINB_>
+template <typename V, int NW_, int K_, int STAGES_, int MINB_, int PFW_ = 0>
 struct CfgK {
     static constexpr bool ROWK = true;
+    static constexpr int PFW = PFW_;                     // x prefetch warps (0 or 1)
     static constexpr int NW = NW_;
     static constexpr int K = K_;
     static constexpr int WSPAN = 32 * K;
     static constexpr int T = NW * WSPAN;
     static constexpr int STAGES = STAGES_;
     static constexpr int MINB = MINB_;
-    static constexpr int THREADS = (NW + 2) * 32;
+    static constexpr int THREADS = (NW + 2 + PFW) * 32;
     static constexpr int RING = 8;
     static constexpr int DATA_BYTES = int(((4 + sizeof(V)) * T + 64 + 15) / 16 * 16);
     static constexpr int FW = (T + 31) / 32 + 1;         // +1: lane masks read two words
@@ -234,7 +236,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
     if (tid == 0) {
         for (int s = 0; s < C::STAGES; ++s) {
             mbar_init(&full[s], 1);
-            mbar_init(&empty[s], NW + 1);
+            mbar_init(&empty[s], NW + 1 + C::PFW);
         }
         for (int s = 0; s < C::RSLOTS; ++s) {
             mbar_init(&rowsrdy[s], 1);
@@ -338,6 +340,27 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                 mbar_arrive(&rowsrdy[rs]);
                 mbar_arrive(&empty[stage]);  // this warp no longer reads the stage
             }
+        }
+    } else if (C::PFW > 0 && warp == NW + 2) {
+        // ============================ x prefetch warp ==========================
+        // As soon as a tile lands -- while the workers still walk the previous
+        // tile -- pull the x lines its columns reference into L1, so the
+        // workers' gathers of that tile hit L1 instead of waiting on L2 while
+        // they hold the stage (the stage hold time bounds the TMA stream).
+        for (int t = 0; t < ntiles; ++t) {
+            const int stage = t % C::STAGES;
+            mbar_wait(&full[stage], (t / C::STAGES) & 1);
+            const int z = meta[stage].j_e - meta[stage].j_s;
+            const int32_t *cs =
+                reinterpret_cast<const int32_t *>(stages + size_t(stage) * C::STAGE_BYTES + meta[stage].col_first);
+            const unsigned col_lim = unsigned(n_cols);
+#pragma unroll 4
+            for (int q = lane; q < z; q += 32) {
+                const unsigned c = unsigned(cs[q]);
+                if (c < col_lim) asm volatile("prefetch.global.L1 [%0];" ::"l"(x + c));
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[stage]);
         }
     } else if constexpr (C::ROWK) {
         // ===================== worker warps (row-aligned) =====================
@@ -718,6 +741,12 @@ msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t
     msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), C::SMEM, "spmv: smem", C::THREADS, &occ);
     if (st != MSP_OK) return st;
     if (occ > 4) occ = 4;
+    static bool said = false;
+    if (!said && getenv("MSP_VERBOSE")) {
+        fprintf(stderr, "msp spmv: rowk=%d K=%d NW=%d PFW=%d T=%d stages=%d smem=%d occupancy=%d CTAs/SM\n", int(C::ROWK),
+                C::K, C::NW, C::PFW, C::T, C::STAGES, C::SMEM, occ);
+        said = true;
+    }
     if (A->nrows == 0) return MSP_OK;
     if (A->nnz == 0)  // every row is empty: y = +0.0 (Z6)
         return cuda_check(cudaMemsetAsync(y, 0, size_t(A->nrows) * sizeof(V), s), "spmv: zero y");
@@ -773,19 +802,36 @@ int nw_choice()
     return nw;
 }
 
-template <typename V, int NW>
-msp_status launch_k(int K, const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
+int pf_choice()
+{
+    static int pf = -1;
+    if (pf < 0) {
+        const char *e = getenv("MSP_SPMV_PF");
+        pf = (e && atoi(e) == 0) ? 0 : 1;
+    }
+    return pf;
+}
+
+template <typename V, int NW, int PF>
+msp_status launch_kp(int K, const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
 {
     constexpr int MB = NW == 4 ? 2 : 1;
     switch (K) {
-    case 7: return launch_cfg<V, CfgK<V, NW, 7, 2, MB>>(A, x, y, ws, ws_bytes, s);
-    case 11: return launch_cfg<V, CfgK<V, NW, 11, 2, MB>>(A, x, y, ws, ws_bytes, s);
-    case 15: return launch_cfg<V, CfgK<V, NW, 15, 2, MB>>(A, x, y, ws, ws_bytes, s);
-    case 19: return launch_cfg<V, CfgK<V, NW, 19, 2, MB>>(A, x, y, ws, ws_bytes, s);
-    case 23: return launch_cfg<V, CfgK<V, NW, 23, 2, MB>>(A, x, y, ws, ws_bytes, s);
-    case 27: return launch_cfg<V, CfgK<V, NW, 27, 2, MB>>(A, x, y, ws, ws_bytes, s);
-    default: return launch_cfg<V, CfgK<V, NW, 31, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    case 7: return launch_cfg<V, CfgK<V, NW, 7, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
+    case 11: return launch_cfg<V, CfgK<V, NW, 11, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
+    case 15: return launch_cfg<V, CfgK<V, NW, 15, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
+    case 19: return launch_cfg<V, CfgK<V, NW, 19, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
+    case 23: return launch_cfg<V, CfgK<V, NW, 23, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
+    case 27: return launch_cfg<V, CfgK<V, NW, 27, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
+    default: return launch_cfg<V, CfgK<V, NW, 31, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
     }
+}
+
+template <typename V, int NW>
+msp_status launch_k(int K, const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
+{
+    return pf_choice() ? launch_kp<V, NW, 1>(K, A, x, y, ws, ws_bytes, s)
+                       : launch_kp<V, NW, 0>(K, A, x, y, ws, ws_bytes, s);
 }
 
 template <typename V>

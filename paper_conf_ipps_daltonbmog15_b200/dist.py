@@ -9,10 +9,13 @@ NVLink/NVSwitch on GPUs; gloo in the CPU tests of the exchange logic).
   x on every rank (the exchange step), then the rank's block of A runs the
   merge-path SpMV locally.  y stays distributed by row blocks.
 * SpGEMM: the row blocks of B are replicated with `gather_csr_blocks`
-  (sizes all-gathered, then one broadcast per source rank straight into its
-  place in the full arrays, offsets rebased on the device); the local
-  symbolic / numeric phases run on the rank's rows of A; `gather_csr_blocks`
-  also concatenates C's row blocks when a replicated C is wanted.
+  (sizes all-gathered, then one padded all-gather per CSR array -- three
+  collectives at any world size -- and a device-side concatenation with the
+  offsets rebased); the local symbolic / numeric phases run on the rank's
+  rows of A; `gather_csr_blocks` also concatenates C's row blocks when a
+  replicated C is wanted (C may instead stay distributed by row blocks).
+* `block_view` / `concat_blocks` are the zero-copy row-block views and the
+  concatenation used on one device (the P-block parity tests).
 
 Compute happens in libmsp kernels (CUDA tensors); only data movement and
 offset rebasing are done here.  CPU tensors are accepted so that the exchange
@@ -78,40 +81,89 @@ def x_slice_of(x_full: torch.Tensor, rank: int, world: int) -> torch.Tensor:
     return s
 
 
+def _all_gather_padded(t: torch.Tensor, n_max: int, group=None) -> torch.Tensor:
+    """Every rank's `t` padded to n_max entries -> [world * n_max] (one
+    collective: all_gather_into_tensor on NCCL, a list all-gather on gloo)."""
+    world = dist.get_world_size(group)
+    pad = torch.zeros(n_max, dtype=t.dtype, device=t.device)
+    pad[:t.numel()] = t
+    out = torch.empty(world * n_max, dtype=t.dtype, device=t.device)
+    if t.is_cuda:
+        dist.all_gather_into_tensor(out, pad, group=group)
+    else:
+        dist.all_gather(list(out.chunk(world)), pad, group=group)
+    return out
+
+
 def gather_csr_blocks(blk: CsrTensor, group=None) -> CsrTensor:
     """Row blocks (in rank order) of a matrix -> the full matrix on every rank.
-    Sizes are all-gathered first; each rank then broadcasts its block into its
-    place in the full arrays; row offsets are rebased by the running nnz."""
+    Block sizes are all-gathered first; then ONE padded all-gather per array
+    (row offsets, columns, values: three collectives whatever the world
+    size) and a device-side concatenation, with each block's offsets rebased
+    by the running nnz (msp_rebase_offsets)."""
     world = dist.get_world_size(group)
     dev = blk.val.device
     meta = torch.tensor([blk.shape[0], blk.nnz], dtype=torch.int64, device=dev)
-    metas = [torch.empty_like(meta) for _ in range(world)]
-    dist.all_gather(metas, meta, group=group)
-    rows = [int(t[0]) for t in metas]
-    nnzs = [int(t[1]) for t in metas]
+    metas = _all_gather_padded(meta, 2, group).view(world, 2).cpu().numpy()
+    rows = [int(r) for r in metas[:, 0]]
+    nnzs = [int(z) for z in metas[:, 1]]
     m, nnz = sum(rows), sum(nnzs)
+    mr, mz = max(rows) + 1, max(max(nnzs), 1)
+    rp_all = _all_gather_padded(blk.rp, mr, group).view(world, mr)
+    col_all = _all_gather_padded(blk.col, mz, group).view(world, mz)
+    val_all = _all_gather_padded(blk.val, mz, group).view(world, mz)
+    return concat_blocks([CsrTensor(rp_all[q, :rows[q] + 1], col_all[q, :nnzs[q]], val_all[q, :nnzs[q]],
+                                    (rows[q], blk.shape[1])) for q in range(world)])
+
+
+def concat_blocks(blocks) -> CsrTensor:
+    """Row blocks (each with offsets starting at 0) -> one CSR matrix: columns
+    and values concatenated, offsets rebased by the running nnz on the
+    device (msp_rebase_offsets).  Used for B replication and for C."""
+    dev = blocks[0].val.device
+    m = sum(b.shape[0] for b in blocks)
+    nnz = sum(b.nnz for b in blocks)
     rp = torch.empty(m + 1, dtype=torch.int32, device=dev)
     col = torch.empty(nnz, dtype=torch.int32, device=dev)
-    val = torch.empty(nnz, dtype=blk.val.dtype, device=dev)
-    r_off = np.concatenate([[0], np.cumsum(rows)]).astype(np.int64)
-    z_off = np.concatenate([[0], np.cumsum(nnzs)]).astype(np.int64)
-    me = dist.get_rank(group)
-    for src in range(world):
-        rsl = slice(int(r_off[src]), int(r_off[src + 1]) + 1)
-        zsl = slice(int(z_off[src]), int(z_off[src + 1]))
-        if src == me:
-            rp_part = _rebase(blk.rp, int(z_off[src]))
-            col[zsl].copy_(blk.col)
-            val[zsl].copy_(blk.val)
-        else:
-            rp_part = torch.empty(rows[src] + 1, dtype=torch.int32, device=dev)
-        gsrc = dist.get_global_rank(group, src) if group is not None else src
-        dist.broadcast(rp_part, gsrc, group=group)
-        if nnzs[src]:
-            dist.broadcast(col[zsl], gsrc, group=group)
-            dist.broadcast(val[zsl], gsrc, group=group)
-        rp[rsl] = rp_part  # already rebased by its source
-    return CsrTensor(rp, col, val, (m, blk.shape[1]))
+    val = torch.empty(nnz, dtype=blocks[0].val.dtype, device=dev)
+    r = z = 0
+    for b in blocks:
+        rp[r:r + b.shape[0] + 1] = _rebase(b.rp.contiguous(), z)
+        col[z:z + b.nnz] = b.col
+        val[z:z + b.nnz] = b.val
+        r += b.shape[0]
+        z += b.nnz
+    if not blocks or m == 0:
+        rp.zero_()
+    return CsrTensor(rp, col, val, (m, blocks[0].shape[1]))
+
+
+def block_view(A: CsrTensor, r0: int, r1: int) -> CsrTensor:
+    """Rows [r0, r1) of a device CSR matrix as a zero-copy block: columns and
+    values are views into A's arrays, only the m_r + 1 row offsets are
+    rebased to start at 0 (msp_rebase_offsets)."""
+    rp_h = A.rp[r0:r1 + 1]
+    a0, a1 = int(A.rp[r0]), int(A.rp[r1])
+    return CsrTensor(_rebase(rp_h.contiguous(), 0), A.col[a0:a1], A.val[a0:a1], (r1 - r0, A.shape[1]))
+
+
+def split_rows_by_products(A_rp_host, A_col_host, B_rp_host, world: int) -> np.ndarray:
+    """Row blocks balanced by SpGEMM products (sum over a row's nonzeros of
+    the referenced B row lengths) instead of by nonzeros: the same
+    lower-bound split (msp_row_split) over the per-row product prefix sum."""
+    bl = np.diff(np.asarray(B_rp_host, dtype=np.int64))
+    w = bl[np.asarray(A_col_host, dtype=np.int64)]
+    cs = np.concatenate([[0], np.cumsum(w)])
+    rp = np.asarray(A_rp_host, dtype=np.int64)
+    prow = cs[rp]  # products before each row
+    m = rp.size - 1
+    total = int(prow[-1])
+    starts = np.empty(world + 1, dtype=np.int32)
+    starts[0], starts[world] = 0, m
+    for r in range(1, world):
+        starts[r] = int(np.searchsorted(prow, -(-r * total // world), side="left"))
+        starts[r] = min(max(starts[r], starts[r - 1]), m)
+    return starts
 
 
 def dist_spmv(A_blk: CsrTensor, x_slice: torch.Tensor, n: int, group=None):

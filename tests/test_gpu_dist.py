@@ -51,3 +51,41 @@ def test_dist_world1(pg):
     assert np.array_equal(rp, W.rp) and np.array_equal(col, W.col)
     ok, msg = oracle.check_values(val, W.val, sc, np.float64)
     assert ok, msg
+
+
+@pytest.mark.parametrize("cfg,scale", [("C4", 0.2), ("C5", 0.005)])
+@pytest.mark.parametrize("P", [2, 4, 8])
+def test_row_blocks_one_gpu(cfg, scale, P):
+    """The multi-GPU decomposition run on one GPU: P nnz-balanced row blocks
+    (zero-copy views with rebased offsets), libmsp SpMV and SpGEMM on each
+    block against the replicated x / B, blocks concatenated -- y, and C's
+    row_offsets / col_idx / values, must equal the oracle's single result bit
+    for bit (integer mode, SURVEY §8(e) correctness)."""
+    from paper_conf_ipps_daltonbmog15_b200 import SpGemmPlan, spmv
+    from paper_conf_ipps_daltonbmog15_b200 import dist as mdist
+    from tests.gpu_util import dev
+    A = gen.config(cfg, "int", scale=scale)
+    x = gen.x_vector(A.n, "int")
+    Ad = dev(A)
+    xd = torch.as_tensor(x, device="cuda")
+    W, _, _ = oracle.spgemm(A, A)
+    yw, _ = oracle.spmv(A, x)
+    for split in ("nnz", "products"):
+        starts = (mdist.split_rows(A.rp, P) if split == "nnz"
+                  else mdist.split_rows_by_products(A.rp, A.col, A.rp, P))
+        assert starts[0] == 0 and starts[-1] == A.m and np.all(np.diff(starts) >= 0)
+        ys, Cs = [], []
+        for r in range(P):
+            blk = mdist.block_view(Ad, int(starts[r]), int(starts[r + 1]))
+            ys.append(spmv(blk, xd))
+            p = SpGemmPlan(blk, Ad)
+            p.setup()
+            p.symbolic()
+            Cs.append(p.numeric())
+        y = torch.cat(ys).cpu().numpy()
+        assert np.array_equal(y, yw), f"{cfg} P={P} {split}: y"
+        C = mdist.concat_blocks(Cs)
+        rp, col, val = C.numpy()
+        assert np.array_equal(rp, W.rp), f"{cfg} P={P} {split}: row_offsets"
+        assert np.array_equal(col, W.col), f"{cfg} P={P} {split}: col_idx"
+        assert np.array_equal(val, W.val), f"{cfg} P={P} {split}: values"
