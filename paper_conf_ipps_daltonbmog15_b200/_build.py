@@ -17,8 +17,8 @@ from pathlib import Path
 PKG = Path(__file__).resolve().parent
 CSRC = PKG / "csrc"
 ROOT = PKG.parent
-LIB = PKG / "libmsp.so"
-BUILD = ROOT / "build" / "msp"
+LIB = Path(os.environ.get("MSP_LIB_OUT", PKG / "libmsp.so"))  # experiment builds may go elsewhere
+BUILD = Path(os.environ.get("MSP_BUILD_DIR", ROOT / "build" / "msp"))
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]

@@ -62,6 +62,8 @@ msp_status scan_widths_to_S(const int32_t *Acol, const int32_t *Brp, int64_t nnz
 // ---------------------------------------------------------------- ops ----
 size_t spmv_ws_bytes(const msp_csr *A);
 msp_status spmv_run(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s);
+// warp-tile row-aligned SpMV (spmv_wt.cu), K odd in 15..31
+msp_status spmv_wt_run(int K, const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s);
 
 size_t spadd_ws_bytes(const msp_csr *A, const msp_csr *B);
 msp_status spadd_symbolic_run(const msp_csr *A, const msp_csr *B, int32_t *Crp, int64_t *nnzC, void *ws,

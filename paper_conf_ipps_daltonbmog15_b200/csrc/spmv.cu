@@ -39,6 +39,24 @@
 #include "common.cuh"
 #include "internal.h"
 
+#ifdef MSP_SPMV_TRACE
+// Timeline instrumentation (experiment builds only): clock64 stamps per
+// (CTA < 4, tile < 64, slot < 16), relative to the CTA's start.
+__device__ long long g_spmv_trace[4][64][16];
+extern "C" int msp_debug_spmv_trace(void *host)
+{
+    return int(cudaMemcpyFromSymbol(host, g_spmv_trace, sizeof(g_spmv_trace)));
+}
+#define TR(t, slot)                                                                                   \
+    do {                                                                                              \
+        if (blockIdx.x < 4 && (t) < 64) g_spmv_trace[blockIdx.x][(t)][(slot)] = clock64() - tr_t0;    \
+    } while (0)
+#else
+#define TR(t, slot) \
+    do {            \
+    } while (0)
+#endif
+
 namespace msp {
 namespace {
 
@@ -63,7 +81,6 @@ struct CtaRecord {  // one per CTA in the workspace
 template <typename V, int NW_, int STAGES_, int RSLOTS_, int MINB_>
 struct Cfg {
     static constexpr bool ROWK = false;
-    static constexpr int PFW = 0;                        // x prefetch warps
     static constexpr int NW = NW_;
     static constexpr int K = 8;
     static constexpr int WSPAN = 32 * K;                 // products per worker warp
@@ -91,28 +108,28 @@ struct Cfg {
 // when rows are about K long, gather u of the 32 lanes touches the same
 // stencil position of 32 consecutive rows -- a few x cache lines per
 // instruction instead of one per row.
-template <typename V, int NW_, int K_, int STAGES_, int MINB_, int PFW_ = 0>
+template <typename V, int NW_, int K_, int STAGES_, int MINB_>
 struct CfgK {
     static constexpr bool ROWK = true;
-    static constexpr int PFW = PFW_;                     // x prefetch warps (0 or 1)
     static constexpr int NW = NW_;
     static constexpr int K = K_;
     static constexpr int WSPAN = 32 * K;
     static constexpr int T = NW * WSPAN;
     static constexpr int STAGES = STAGES_;
     static constexpr int MINB = MINB_;
-    static constexpr int THREADS = (NW + 2 + PFW) * 32;
+    static constexpr int THREADS = (NW + 2) * 32;
     static constexpr int RING = 8;
     static constexpr int DATA_BYTES = int(((4 + sizeof(V)) * T + 64 + 15) / 16 * 16);
-    static constexpr int FW = (T + 31) / 32 + 1;         // +1: lane masks read two words
-    static constexpr int FLAG_BYTES = (FW * 4 + 15) / 16 * 16;
-    static constexpr int RMAP_BYTES = (T * 2 + 15) / 16 * 16;
+    static constexpr int FW = 1;
     static constexpr int STAGE_BYTES = DATA_BYTES;
-    static constexpr int RSLOTS = STAGES_;
-    static constexpr int RSLOT_BYTES = FLAG_BYTES + RMAP_BYTES;
-    static constexpr int PROD_BYTES = 0;
+    static constexpr int RSLOTS = 0;                     // no shared row map: each worker maps its own span
+    static constexpr int RSLOT_BYTES = 0;
+    // per worker warp: 32 lane masks of row-end bits + the tile-relative row
+    // id at every row-end position of its span (WSPAN 16-bit entries)
+    static constexpr int WMAP_BYTES = (32 * 4 + WSPAN * 2 + 15) / 16 * 16;
+    static constexpr int PROD_BYTES = NW * WMAP_BYTES;
     static constexpr int MISC_BYTES = 2048;
-    static constexpr int SMEM = STAGES * STAGE_BYTES + RSLOTS * RSLOT_BYTES + PROD_BYTES + MISC_BYTES;
+    static constexpr int SMEM = STAGES * STAGE_BYTES + PROD_BYTES + MISC_BYTES;
     static_assert(K % 2 == 1 && K < 32, "K odd and < 32");
 };
 
@@ -162,6 +179,18 @@ __device__ __forceinline__ double ldg_x(const float *p)
     return double(v);
 }
 
+// Predicated global store (keeps the walk straight-line code).
+__device__ __forceinline__ void st_global_if(double *p, double v, bool pred)
+{
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.f64 [%0], %1;\n\t}" ::"l"(p), "d"(v),
+                 "r"(int(pred)));
+}
+__device__ __forceinline__ void st_global_if(float *p, float v, bool pred)
+{
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %2, 0;\n\t@p st.global.f32 [%0], %1;\n\t}" ::"l"(p), "f"(v),
+                 "r"(int(pred)));
+}
+
 __device__ __forceinline__ void mbar_wait_backoff(uint64_t *bar, uint32_t parity)
 {
     while (!mbar_try_wait(bar, parity)) {
@@ -208,6 +237,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
     char *stages = smem;
     char *rslots = smem + C::STAGES * C::STAGE_BYTES;                   // [RSLOTS] flags + row map
     double *prodbuf = reinterpret_cast<double *>(rslots + C::RSLOTS * C::RSLOT_BYTES);  // [NW][WSPAN]
+    char *prodbuf_raw = reinterpret_cast<char *>(prodbuf);  // row-aligned variant: [NW] warp row maps
     char *misc = reinterpret_cast<char *>(prodbuf) + C::PROD_BYTES;
     uint64_t *full = reinterpret_cast<uint64_t *>(misc);               // [STAGES] TMA landed
     uint64_t *empty = full + C::STAGES;                                // [STAGES] stage free
@@ -229,6 +259,9 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
     const int warp = tid >> 5;
     const int G = gridDim.x;
     const int64_t total = int64_t(m) + nnz;
+#ifdef MSP_SPMV_TRACE
+    const long long tr_t0 = clock64();
+#endif
     const int64_t d_begin = int64_t(blockIdx.x) * total / G;
     const int64_t d_end = int64_t(blockIdx.x + 1) * total / G;
     const int ntiles = int((d_end - d_begin + C::T - 1) / C::T);
@@ -236,7 +269,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
     if (tid == 0) {
         for (int s = 0; s < C::STAGES; ++s) {
             mbar_init(&full[s], 1);
-            mbar_init(&empty[s], NW + 1 + C::PFW);
+            mbar_init(&empty[s], NW + 1);
         }
         for (int s = 0; s < C::RSLOTS; ++s) {
             mbar_init(&rowsrdy[s], 1);
@@ -268,7 +301,9 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             const int i_e = warp_grid_search_guess(rp, de, lo, hi, i_s + prev_rows, lane);
             const int j_e = int(de - i_e);
             prev_rows = i_e - i_s;
+            if (lane == 0) TR(t, 0);  // split searched
             if (t >= C::STAGES) mbar_wait_backoff(&empty[stage], ((t / C::STAGES) - 1) & 1);
+            if (lane == 0) TR(t, 1);  // stage free: TMA issued
             char *sb = stages + size_t(stage) * C::STAGE_BYTES;
             const int wr_end = min(i_e + 1, m);
             // windows: rp[i_s .. wr_end] (inclusive), col/val[j_s .. j_e)
@@ -306,10 +341,38 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
         // position of every nonempty row's last nonzero; empty rows whose
         // row-end item lies in the tile get y = +0.0 (Z6); the row holding the
         // tile's last nonzero is the CTA carry key.
+        if constexpr (C::ROWK) {
+            // row-aligned workers map their own spans' row ends: this warp only
+            // zero-fills the tile's empty rows (Z6) and tracks the carry key
+            for (int t = 0; t < ntiles; ++t) {
+                const int stage = t % C::STAGES;
+                mbar_wait(&full[stage], (t / C::STAGES) & 1);
+                if (lane == 0) TR(t, 2);  // landed (row warp)
+                const TileMeta mt = meta[stage];
+                const int32_t *rps = reinterpret_cast<const int32_t *>(stages + size_t(stage) * C::STAGE_BYTES +
+                                                                       mt.rp_first);
+                const int z = mt.j_e - mt.j_s, i_s = mt.i_s, j_s = mt.j_s;
+                for (int r = i_s + lane; r < mt.wr_end; r += 32) {
+                    const int a = rps[r - i_s] - j_s;
+                    const int b = rps[r - i_s + 1] - j_s;
+                    if (a == b) {
+                        if (r < mt.i_e) y[r] = V(0);
+                    } else if (z > 0 && a < z && b >= z) {
+                        s_carry_key = (b > z) ? r : -1;
+                    }
+                }
+                __syncwarp();
+                if (lane == 0) {
+                    TR(t, 3);
+                    mbar_arrive(&empty[stage]);  // this warp no longer reads the stage
+                }
+            }
+        } else
         for (int t = 0; t < ntiles; ++t) {
             const int stage = t % C::STAGES;
             const int rs = t % C::RSLOTS;
             mbar_wait(&full[stage], (t / C::STAGES) & 1);
+            if (lane == 0) TR(t, 2);  // landed (row warp)
             if (t >= C::RSLOTS) mbar_wait(&rowsfree[rs], ((t / C::RSLOTS) - 1) & 1);
             const TileMeta mt = meta[stage];
             char *sb = stages + size_t(stage) * C::STAGE_BYTES;
@@ -337,30 +400,10 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             }
             __syncwarp();
             if (lane == 0) {
+                TR(t, 3);  // row map built
                 mbar_arrive(&rowsrdy[rs]);
                 mbar_arrive(&empty[stage]);  // this warp no longer reads the stage
             }
-        }
-    } else if (C::PFW > 0 && warp == NW + 2) {
-        // ============================ x prefetch warp ==========================
-        // As soon as a tile lands -- while the workers still walk the previous
-        // tile -- pull the x lines its columns reference into L1, so the
-        // workers' gathers of that tile hit L1 instead of waiting on L2 while
-        // they hold the stage (the stage hold time bounds the TMA stream).
-        for (int t = 0; t < ntiles; ++t) {
-            const int stage = t % C::STAGES;
-            mbar_wait(&full[stage], (t / C::STAGES) & 1);
-            const int z = meta[stage].j_e - meta[stage].j_s;
-            const int32_t *cs =
-                reinterpret_cast<const int32_t *>(stages + size_t(stage) * C::STAGE_BYTES + meta[stage].col_first);
-            const unsigned col_lim = unsigned(n_cols);
-#pragma unroll 4
-            for (int q = lane; q < z; q += 32) {
-                const unsigned c = unsigned(cs[q]);
-                if (c < col_lim) asm volatile("prefetch.global.L1 [%0];" ::"l"(x + c));
-            }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&empty[stage]);
         }
     } else if constexpr (C::ROWK) {
         // ===================== worker warps (row-aligned) =====================
@@ -371,7 +414,9 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
         // earlier lanes); the warp segmented scan and the look-back across
         // warps / tiles are the same as in the transpose variant below.
         const int q0 = warp * WSPAN + lane * K;
-        const int fw0 = q0 >> 5, fsh = q0 & 31;
+        const int sp0 = warp * WSPAN;  // the warp's span of tile positions [sp0, sp0 + WSPAN)
+        uint32_t *wmask = reinterpret_cast<uint32_t *>(prodbuf_raw + size_t(warp) * C::WMAP_BYTES);  // [32]
+        uint16_t *wrow = reinterpret_cast<uint16_t *>(wmask + 32);  // [WSPAN] tile-relative row per row end
         auto finish_first = [&](int r, double v0, int tt) {
             const int sl = tt & (RING - 1);
             double c = 0.0;
@@ -401,49 +446,133 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
         for (int t = 0; t < ntiles; ++t) {
             const int stage = t % C::STAGES;
             const int slot = t & (RING - 1);
-            const int rs = t % C::RSLOTS;
             mbar_wait(&full[stage], (t / C::STAGES) & 1);
-            const int tile_is = meta[stage].i_s;
-            const int z = meta[stage].j_e - meta[stage].j_s;
+            if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 8 : 4);  // worker sees the stage
+            const TileMeta mt = meta[stage];
+            const int tile_is = mt.i_s;
+            const int z = mt.j_e - mt.j_s;
             const char *sb = stages + size_t(stage) * C::STAGE_BYTES;
-            const int32_t *cs = reinterpret_cast<const int32_t *>(sb + meta[stage].col_first);
-            const V *vs = reinterpret_cast<const V *>(sb + meta[stage].val_first);
+            const int32_t *cs = reinterpret_cast<const int32_t *>(sb + mt.col_first);
+            const V *vs = reinterpret_cast<const V *>(sb + mt.val_first);
+            const int32_t *rps = reinterpret_cast<const int32_t *>(sb + mt.rp_first);  // rps[k] = rp[i_s + k]
             // ---- gathers: K independent loads in flight per lane ----
+            // all column reads first (plain shared loads, issued back to back),
+            // then the K gathers: the volatile gathers keep program order, so
+            // interleaving them with the column reads would serialise one
+            // shared-memory latency per gather.  Positions >= z gather x[0]
+            // (their products are masked in the walk).
+            int cidx[K];
+#pragma unroll
+            for (int u = 0; u < K; ++u) cidx[u] = (q0 + u < z) ? cs[q0 + u] : 0;
             double xv[K];
 #pragma unroll
-            for (int u = 0; u < K; ++u) {
-                const int q = q0 + u;
-                xv[u] = 0.0;
-                if (q < z) xv[u] = ldg_x(x + cs[q]);
-            }
-            mbar_wait(&rowsrdy[rs], (t / C::RSLOTS) & 1);
-            const uint32_t *flags = reinterpret_cast<const uint32_t *>(rslots + size_t(rs) * C::RSLOT_BYTES);
-            const uint16_t *rmap =
-                reinterpret_cast<const uint16_t *>(rslots + size_t(rs) * C::RSLOT_BYTES + C::FLAG_BYTES);
-            const unsigned mask = __funnelshift_r(flags[fw0], flags[fw0 + 1], fsh) & ((1u << K) - 1u);
-            // ---- walk ----
-            double run = 0.0, first_v = 0.0;
-            int first_k = -1;
+            for (int u = 0; u < K; ++u) xv[u] = ldg_x(x + cidx[u]);
+            // values into registers while the gathers fly (one burst of
+            // conflict-free shared loads; the walk then reads registers only)
+            double vv[K];
 #pragma unroll
-            for (int u = 0; u < K; ++u) {
-                const int q = q0 + u;
-                if (q < z) run = fma(double(vs[q]), xv[u], run);
-                if ((mask >> u) & 1u) {
-                    if (first_k < 0) {
-                        first_k = u;
-                        first_v = run;
-                    } else {
-                        y[tile_is + int(rmap[q]) - 1] = V(run);
+            for (int u = 0; u < K; ++u) vv[u] = double(vs[q0 + u]);
+            if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 9 : 5);  // gathers issued
+            // ---- this warp's row ends (no shared row warp: warps never wait
+            //      on each other's maps) ----
+            // Row k of the tile (global i_s + k) ends at tile position
+            // e_k = rps[k+1] - j_s; a nonempty row is emitted at its last
+            // nonzero e_k - 1 if that lies in [0, z) (empty rows: row warp).
+            const int sp1 = min(sp0 + WSPAN, z);
+            wmask[lane] = 0u;
+            __syncwarp();
+            if (sp0 < sp1) {
+                const int nwin = mt.wr_end - mt.i_s;  // rows in the window
+                const int j_s = mt.j_s;
+                // first row ending after sp0: 32-ary search over the window
+                int lo = 0, hi = nwin;
+                while (hi - lo > 32) {
+                    const int step = (hi - lo + 31) >> 5;
+                    const int pp = lo + (lane + 1) * step - 1;
+                    const bool pr = pp < hi && rps[pp + 1] - j_s <= sp0;
+                    const int c = __popc(__ballot_sync(0xffffffffu, pr));
+                    const int nhi = min(hi, lo + (c + 1) * step - 1);
+                    lo = lo + c * step;
+                    hi = c < 32 ? nhi : hi;
+                }
+                {
+                    const int pp = lo + lane;
+                    const bool pr = pp < hi && rps[pp + 1] - j_s <= sp0;
+                    lo += __popc(__ballot_sync(0xffffffffu, pr));
+                }
+                for (int k = lo + lane;; k += 32) {
+                    int e = INT_MAX, a = 0;
+                    if (k < nwin) {
+                        a = rps[k] - j_s;
+                        e = rps[k + 1] - j_s;
                     }
-                    run = 0.0;
+                    if (e <= sp1 && a < e) {  // nonempty row ending in the span
+                        const int pos = e - 1 - sp0;
+                        const int ol = pos / K, bit = pos - ol * K;
+                        atomicOr(&wmask[ol], 1u << bit);
+                        wrow[pos] = uint16_t(k);
+                    }
+                    if (!__any_sync(0xffffffffu, e < sp1)) break;
                 }
             }
-            const int first_r = first_k >= 0 ? tile_is + int(rmap[q0 + first_k]) - 1 : -1;
             __syncwarp();
-            if (lane == 0) {  // stage and row map of this tile no longer read by this warp
+            const unsigned mask = wmask[lane];
+            __syncwarp();
+            if (lane == 0) {  // cols, vals and row offsets of this tile are in registers / the warp map now
+                if (warp == 0 || warp == NW - 1) TR(t, warp ? 13 : 12);  // own map built
                 mbar_arrive(&empty[stage]);
-                mbar_arrive(&rowsfree[rs]);
             }
+#ifdef MSP_SPMV_TRACE
+            asm volatile("" ::"d"(xv[K - 1]));
+            if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 15 : 14);  // last gather returned
+#endif
+            // ---- walk (branch-free) ----
+            // Every step is straight-line code: the multiply-add, the row-end
+            // bit, a select that keeps the first row end's partial (it needs
+            // the carry of earlier lanes, below), a predicated store for every
+            // later row end, and a select that restarts the running sum.
+            const int first_k = mask ? __ffs(mask) - 1 : K;
+            V *ybase = y + tile_is;
+            const uint16_t *lrow = wrow + lane * K;
+            double run = 0.0, first_v = 0.0;
+            auto walk = [&](auto tail) {
+#pragma unroll
+                for (int u = 0; u < K; ++u) {
+                    double v = vv[u];
+                    if constexpr (decltype(tail)::value) v = (q0 + u < z) ? v : 0.0;  // partial last tile
+                    run = fma(v, xv[u], run);
+                    const bool b = (mask >> u) & 1u;
+                    first_v = (u == first_k) ? run : first_v;
+                    const bool later = b && (u > first_k);
+                    const int rr = later ? int(lrow[u]) : 0;
+                    st_global_if(ybase + rr, V(run), later);
+                    run = b ? 0.0 : run;
+                }
+            };
+#ifdef MSP_SPMV_BRANCHY_WALK  // experiment: the round-1 walk (a branch per row end)
+            (void)walk;
+            {
+                int fk = -1;
+#pragma unroll
+                for (int u = 0; u < K; ++u) {
+                    if (q0 + u < z) run = fma(vv[u], xv[u], run);
+                    if ((mask >> u) & 1u) {
+                        if (fk < 0) {
+                            fk = u;
+                            first_v = run;
+                        } else {
+                            ybase[lrow[u]] = V(run);
+                        }
+                        run = 0.0;
+                    }
+                }
+            }
+#else
+            if (q0 + K <= z) walk(std::false_type{});
+            else walk(std::true_type{});
+#endif
+            const int first_r = mask ? tile_is + int(lrow[first_k]) : -1;
+            if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 10 : 6);  // walk done
             const bool flagged = first_r >= 0;
             // ---- warp segmented scan ----
             const SegPair<double> inc = warp_seg_inclusive(SegPair<double>{flagged, run}, lane);
@@ -489,6 +618,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                 }
             }
             if (pend_r >= 0) finish_first(pend_r, pend_v, pend_t);
+            if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 11 : 7);  // tile finished
             pend_r = (lane == flane) ? first_r : -1;
             pend_v = pend_nv;
             pend_t = t;
@@ -604,30 +734,20 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                         p[2 * i + 1] = (qs + 2 * i + 1 < z) ? d2.y : 0.0;
                     }
                 }
-                double ev[K];
+                // branch-free walk: predicated stores for every row end after
+                // the lane's first (whose partial waits for the lane carry)
+                const int k0 = mask ? __ffs(mask) - 1 : K;
 #pragma unroll
                 for (int k = 0; k < K; ++k) {
                     run += p[k];
-                    ev[k] = run;
-                    if ((mask >> k) & 1u) run = 0.0;
+                    const bool b = (mask >> k) & 1u;
+                    first_v = (k == k0) ? run : first_v;
+                    const bool later = b && (k > k0);
+                    const int rr = later ? int(rmap[qs + k]) : 1;
+                    st_global_if(y + tile_is + rr - 1, V(run), later);
+                    run = b ? 0.0 : run;
                 }
-                if (mask) {
-                    // pick row partials from registers (no shared-memory round
-                    // trip: the L1/shared data pipe is the kernel's limit)
-                    auto pick = [&](int kk) {
-                        double r = ev[0];
-#pragma unroll
-                        for (int k = 1; k < K; ++k) r = (k == kk) ? ev[k] : r;
-                        return r;
-                    };
-                    const int k0 = __ffs(mask) - 1;
-                    first_v = pick(k0);
-                    first_r = tile_is + int(rmap[qs + k0]) - 1;
-                    for (unsigned rest = mask & (mask - 1); rest; rest &= rest - 1) {
-                        const int k = __ffs(rest) - 1;
-                        y[tile_is + int(rmap[qs + k]) - 1] = V(pick(k));
-                    }
-                }
+                if (mask) first_r = tile_is + int(rmap[qs + k0]) - 1;
             }
             const bool flagged = first_r >= 0;
             // ---- warp segmented scan ----
@@ -743,8 +863,8 @@ msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t
     if (occ > 4) occ = 4;
     static bool said = false;
     if (!said && getenv("MSP_VERBOSE")) {
-        fprintf(stderr, "msp spmv: rowk=%d K=%d NW=%d PFW=%d T=%d stages=%d smem=%d occupancy=%d CTAs/SM\n", int(C::ROWK),
-                C::K, C::NW, C::PFW, C::T, C::STAGES, C::SMEM, occ);
+        fprintf(stderr, "msp spmv: rowk=%d K=%d NW=%d T=%d stages=%d smem=%d occupancy=%d CTAs/SM\n", int(C::ROWK),
+                C::K, C::NW, C::T, C::STAGES, C::SMEM, occ);
         said = true;
     }
     if (A->nrows == 0) return MSP_OK;
@@ -802,36 +922,31 @@ int nw_choice()
     return nw;
 }
 
-int pf_choice()
+// Warp-tile kernel (spmv_wt.cu) for the row-aligned layout; MSP_SPMV_WT=0
+// selects the CTA-tile kernel below (tuning / comparison only).
+int wt_choice()
 {
-    static int pf = -1;
-    if (pf < 0) {
-        const char *e = getenv("MSP_SPMV_PF");
-        pf = (e && atoi(e) == 0) ? 0 : 1;
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("MSP_SPMV_WT");
+        v = (e && atoi(e) == 0) ? 0 : 1;
     }
-    return pf;
-}
-
-template <typename V, int NW, int PF>
-msp_status launch_kp(int K, const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
-{
-    constexpr int MB = NW == 4 ? 2 : 1;
-    switch (K) {
-    case 7: return launch_cfg<V, CfgK<V, NW, 7, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
-    case 11: return launch_cfg<V, CfgK<V, NW, 11, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
-    case 15: return launch_cfg<V, CfgK<V, NW, 15, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
-    case 19: return launch_cfg<V, CfgK<V, NW, 19, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
-    case 23: return launch_cfg<V, CfgK<V, NW, 23, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
-    case 27: return launch_cfg<V, CfgK<V, NW, 27, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
-    default: return launch_cfg<V, CfgK<V, NW, 31, 2, MB, PF>>(A, x, y, ws, ws_bytes, s);
-    }
+    return v;
 }
 
 template <typename V, int NW>
 msp_status launch_k(int K, const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
 {
-    return pf_choice() ? launch_kp<V, NW, 1>(K, A, x, y, ws, ws_bytes, s)
-                       : launch_kp<V, NW, 0>(K, A, x, y, ws, ws_bytes, s);
+    constexpr int MB = NW == 4 ? 2 : 1;
+    switch (K) {
+    case 7: return launch_cfg<V, CfgK<V, NW, 7, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    case 11: return launch_cfg<V, CfgK<V, NW, 11, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    case 15: return launch_cfg<V, CfgK<V, NW, 15, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    case 19: return launch_cfg<V, CfgK<V, NW, 19, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    case 23: return launch_cfg<V, CfgK<V, NW, 23, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    case 27: return launch_cfg<V, CfgK<V, NW, 27, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    default: return launch_cfg<V, CfgK<V, NW, 31, 2, MB>>(A, x, y, ws, ws_bytes, s);
+    }
 }
 
 template <typename V>
@@ -843,6 +958,7 @@ msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_
     switch (shape) {
     case -1: {
         const int K = k_choice(A);
+        if (wt_choice() && K >= 15) return spmv_wt_run(K, A, x, y, ws, ws_bytes, s);
         return nw_choice() == 8 ? launch_k<V, 8>(K, A, x, y, ws, ws_bytes, s)
                                 : launch_k<V, 4>(K, A, x, y, ws, ws_bytes, s);
     }
