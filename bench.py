@@ -350,6 +350,13 @@ def ncu_traffic(world):
         return {"traffic": None, "traffic_source": f"unavailable: {e}"}
 
 
+def spmv_kernel_name(m, nnz):
+    """The SpMV kernel libmsp picks for this matrix: warp tiles
+    with row-aligned lanes when the mean row length is >= 20, else the
+    CTA-tile transpose walk."""
+    return "spmv_wt_kernel" if m > 0 and nnz >= 20 * m else "spmv_merge_kernel"
+
+
 class Timer:
     """CUDA events on the launching stream."""
 
@@ -685,7 +692,7 @@ def msp_arm(args):
                        "l2": "inputs larger than L2 (A = 318 MB per rank > 126 MB); x (8 MB) L2-resident; "
                              "table: L2 flushed between launches for inputs < 2x L2"},
             "ops": ops_out,
-            "roofline": {"bound": "hbm", "kernel": "spmv_merge_kernel", "achieved": achieved, "peak": peak,
+            "roofline": {"bound": "hbm", "kernel": spmv_kernel_name(m_loc, A.nnz), "achieved": achieved, "peak": peak,
                          "peak_kind": peak_kind, "unit": "GB/s", "frac": achieved / peak,
                          "alg_bytes_per_launch": by_loc, "launches_timed": len(spmv_kernel_ms),
                          **ncu_traffic(world)},

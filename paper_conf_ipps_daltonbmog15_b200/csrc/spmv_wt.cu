@@ -175,8 +175,8 @@ __device__ __forceinline__ void lb_publish(LbRec *r, double v, int f, int tag)
 template <typename V, class C>
 __global__ void __launch_bounds__(C::THREADS, 1)
 spmv_wt_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const int32_t *__restrict__ col,
-               const V *__restrict__ val, const V *__restrict__ x, V *__restrict__ y, WtRecord *__restrict__ recs,
-               unsigned *__restrict__ counter)
+               const V *__restrict__ val, const V *__restrict__ x, V *__restrict__ y, int32_t n_cols,
+               WtRecord *__restrict__ recs, unsigned *__restrict__ counter)
 {
     constexpr int K = C::K, NW = C::NW, S = C::STAGES, TI = C::TI, RL = C::RL, NSUB = C::NSUB, T = C::T;
     extern __shared__ __align__(128) char smem[];
@@ -336,15 +336,19 @@ spmv_wt_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const int
             const V *vs = reinterpret_cast<const V *>(sb + st.val_first) + j0;
             const int32_t *rps = rpb + i0;  // rps[k] = rp[mt.i_s + k]
             // ---- gathers (K in flight per lane), values into registers ----
+            // positions >= z (the tile's last lanes) read stale slot bytes:
+            // their columns are clamped into x (a valid address) and their
+            // products are masked in the walk (no per-position select here)
+            const unsigned cmax = unsigned(n_cols - 1);
             int cidx[K];
 #pragma unroll
-            for (int u = 0; u < K; ++u) cidx[u] = (q0 + u < z) ? cs[q0 + u] : 0;
+            for (int u = 0; u < K; ++u) cidx[u] = int(min(unsigned(cs[q0 + u]), cmax));
             double xv[K];
 #pragma unroll
             for (int u = 0; u < K; ++u) xv[u] = ldg_xv(x + cidx[u]);
             double vv[K];
 #pragma unroll
-            for (int u = 0; u < K; ++u) vv[u] = double(vs[q0 + u]);  // positions >= z: fixed up below
+            for (int u = 0; u < K; ++u) vv[u] = double(vs[q0 + u]);
             // ---- row ends of the tile -> lane masks + row ids; empty rows ----
             wmask[lane] = 0u;
             __syncwarp();
@@ -374,26 +378,15 @@ spmv_wt_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const int
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[slot]);  // this warp tile of the stage is in regs / the map
             if (lane == 0) WTR(t, 4);  // released
-            // positions past the tile's last product (the last lanes of a tile):
-            // zero product, even if x[0] or the stale slot bytes are not finite
-            // (a divergent branch taken by those lanes only, after the gathers
-            // had the map building to return)
-            if (q0 + K > z) {
-#pragma unroll
-                for (int u = 0; u < K; ++u)
-                    if (q0 + u >= z) {
-                        vv[u] = 0.0;
-                        xv[u] = 0.0;
-                    }
-            }
             // ---- walk: K fp64 multiply-adds, y at each row end ----
             V *ybase = y + mt.i_s;
             const uint16_t *lrow = wrow + q0;
             double run = 0.0, first_v = 0.0;
             int first_k = -1;
+            const int lim = z - q0;  // products of this lane: u < lim
 #pragma unroll
             for (int u = 0; u < K; ++u) {
-                run = fma(vv[u], xv[u], run);
+                if (u < lim) run = fma(vv[u], xv[u], run);
                 if ((mask >> u) & 1u) {
                     if (first_k < 0) {
                         first_k = u;
@@ -407,18 +400,27 @@ spmv_wt_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const int
             const int first_r = first_k >= 0 ? mt.i_s + int(lrow[first_k]) : -1;
             if (lane == 0) WTR(t, 5);  // walked
             const bool flagged = first_r >= 0;
-            // ---- warp segmented scan: carries between lanes ----
-            const SegPair<double> inc = warp_seg_inclusive(SegPair<double>{flagged, run}, lane);
-            const double exv = __shfl_up_sync(0xffffffffu, inc.v, 1);
+            // ---- carries between lanes ----
             const unsigned fmask = __ballot_sync(0xffffffffu, flagged);
+            const unsigned active = __ballot_sync(0xffffffffu, lim > 0);  // lanes 0.. with products
             const int flane = fmask ? __ffs(fmask) - 1 : -1;
+            double exv, agg;
+            if (fmask == active && active) {
+                // every lane with products ends a row (a stencil tile): the
+                // carry into a lane is its left neighbour's trailing sum
+                exv = __shfl_up_sync(0xffffffffu, run, 1);
+                agg = __shfl_sync(0xffffffffu, run, 31 - __clz(active));
+            } else {  // general case: warp segmented scan
+                const SegPair<double> inc = warp_seg_inclusive(SegPair<double>{flagged, run}, lane);
+                exv = __shfl_up_sync(0xffffffffu, inc.v, 1);
+                agg = __shfl_sync(0xffffffffu, inc.v, 31);  // trailing sum of the tile
+            }
             double nv = 0.0;
             if (flagged) {
                 const double v = lane ? first_v + exv : first_v;
                 if (lane == flane) nv = v;
                 else y[first_r] = V(v);
             }
-            const double agg = __shfl_sync(0xffffffffu, inc.v, 31);  // trailing sum of the tile
             if (lane == 0 && fmask) lb_publish(&lb[t & (RL - 1)], agg, 1, ((t + 1) << 2) | 2);  // carry-out known
             else if (lane == 0) lb_publish(&lb[t & (RL - 1)], agg, 0, ((t + 1) << 2) | 1);     // aggregate only
             // ---- finish the previous tile of this warp (deferred look-back) ----
@@ -520,7 +522,7 @@ msp_status launch_wt(const msp_csr *A, const void *x, void *y, void *ws, size_t 
     if (!cv.ok()) return MSP_ERR_WORKSPACE;
     kern<<<grid, C::THREADS, C::SMEM, s>>>(A->nrows, A->nnz, A->row_offsets, A->col_idx,
                                           static_cast<const V *>(A->vals), static_cast<const V *>(x),
-                                          static_cast<V *>(y), recs, counter);
+                                          static_cast<V *>(y), A->ncols, recs, counter);
     return last_launch("spmv_wt_kernel");
 }
 

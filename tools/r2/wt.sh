@@ -1,5 +1,5 @@
 set -x
-D=gpurun_out/${WT_DIR:-wt3}
+D=gpurun_out/${WT_DIR:-wt4}
 mkdir -p $D
 timeout 600 python -m pytest tests/test_gpu_spmv.py -x -q > $D/tests.log 2>&1; echo tests $?
 python tools/spmv_tune.py C2 "CFG=-3" "CFG=-3" "WT=0" > $D/tune.txt 2>&1
