@@ -57,6 +57,16 @@ int sm_count()
     return cache[dev];
 }
 
+// Pinned host words per host thread for the synchronising size read-backs
+// (a pageable destination would stage each small copy through a driver
+// buffer).  Never freed: one small allocation per host thread.
+int64_t *pinned_scratch()
+{
+    static thread_local int64_t *p = nullptr;
+    if (!p && cudaMallocHost(reinterpret_cast<void **>(&p), 16 * sizeof(int64_t)) != cudaSuccess) p = nullptr;
+    return p;
+}
+
 // Large-shared-memory opt-in, once per (device, kernel): the attribute is a
 // per-device property, so a process driving several GPUs sets it on each.
 // Returns the occupancy (resident CTAs per SM) when `threads` > 0.

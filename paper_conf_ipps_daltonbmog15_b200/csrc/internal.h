@@ -20,6 +20,8 @@ int sm_count();
 msp_status cuda_check(cudaError_t e, const char *where);
 msp_status last_launch(const char *where);  // also counts the launch
 uint64_t launch_count();
+// 16 pinned int64 words per host thread (NULL if pinned allocation failed)
+int64_t *pinned_scratch();
 // cudaFuncAttributeMaxDynamicSharedMemorySize (and, with threads > 0, the
 // max carveout + occupancy query) once per (device, kernel).
 msp_status set_smem_attr(const void *func, int smem_bytes, const char *where, int threads = 0, int *occ = nullptr);

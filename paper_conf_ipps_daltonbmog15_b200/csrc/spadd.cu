@@ -473,7 +473,9 @@ msp_status spadd_symbolic_run(const msp_csr *A, const msp_csr *B, int32_t *Crp, 
     if (st != MSP_OK) return st;
     st = scan_i32_to_i64(w.tile_count, w.tile_off, w.ntiles, w.scan, w.scan_bytes, s);
     if (st != MSP_OK) return st;
-    int64_t h[2] = {0, 0};
+    int64_t hbuf[2] = {0, 0};
+    int64_t *pin = pinned_scratch();
+    int64_t *h = pin ? pin : hbuf;
     st = cuda_check(cudaMemcpyAsync(&h[0], &w.totals[0], sizeof(int64_t), cudaMemcpyDeviceToHost, s), "spadd: nnz");
     if (st != MSP_OK) return st;
     st = cuda_check(cudaMemcpyAsync(&h[1], &w.tile_off[w.ntiles], sizeof(int64_t), cudaMemcpyDeviceToHost, s),

@@ -588,8 +588,10 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             // ---- publish the warp's trailing sum; the last warp forms the
             //      carry leaving the tile ----
             if (lane == 31) {
-                agg_v[slot * NW + warp] = inc.v;
-                agg_f[slot * NW + warp] = inc.f;
+                // published through volatile stores, ordered before the tag by
+                // the CTA fence (message passing; readers spin on the tag)
+                reinterpret_cast<volatile double *>(agg_v)[slot * NW + warp] = inc.v;
+                reinterpret_cast<volatile int *>(agg_f)[slot * NW + warp] = inc.f;
                 __threadfence_block();
                 st_volatile_s(&agg_seq[slot * NW + warp], t + 1);
                 const int done = atomicAdd(&pub_cnt[slot], 1);
@@ -610,8 +612,8 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                         c = fw ? vw : c + vw;
                         f |= fw;
                     }
-                    cta_v[slot] = c;
-                    cta_f[slot] = f;
+                    reinterpret_cast<volatile double *>(cta_v)[slot] = c;
+                    reinterpret_cast<volatile int *>(cta_f)[slot] = f;
                     pub_cnt[slot] = 0;
                     __threadfence_block();
                     st_volatile_s(&cta_seq[slot], t + 1);
@@ -766,8 +768,10 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             // ---- publish this warp's trailing sum; the last warp of the tile
             //      forms the carry leaving the tile ----
             if (lane == 31) {
-                agg_v[slot * NW + warp] = inc.v;
-                agg_f[slot * NW + warp] = inc.f;
+                // published through volatile stores, ordered before the tag by
+                // the CTA fence (message passing; readers spin on the tag)
+                reinterpret_cast<volatile double *>(agg_v)[slot * NW + warp] = inc.v;
+                reinterpret_cast<volatile int *>(agg_f)[slot * NW + warp] = inc.f;
                 __threadfence_block();
                 st_volatile_s(&agg_seq[slot * NW + warp], t + 1);
                 const int done = atomicAdd(&pub_cnt[slot], 1);
@@ -788,8 +792,8 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                         c = fw ? vw : c + vw;
                         f |= fw;
                     }
-                    cta_v[slot] = c;
-                    cta_f[slot] = f;
+                    reinterpret_cast<volatile double *>(cta_v)[slot] = c;
+                    reinterpret_cast<volatile int *>(cta_f)[slot] = f;
                     pub_cnt[slot] = 0;
                     __threadfence_block();
                     st_volatile_s(&cta_seq[slot], t + 1);
