@@ -120,6 +120,22 @@ msp_status msp_spmv(const msp_csr *A, const void *x, void *y, void *ws, size_t w
                     void *stream);
 
 /* ------------------------------------------------------------------------
+ * SpMV, the paper's own decomposition (ablation):
+ * a nonzero-only split -- every CTA gets the same number of nonzeros,
+ * Nprods = 2048 -- with the CSR row offsets compacted to the
+ * nonempty rows first, a partition kernel (one binary search
+ * per CTA segment), a reduction kernel (strided loads, x
+ * gathers, strided -> blocked transpose in shared memory, CTA segmented
+ * scan) and an update kernel adding every CTA's (row, partial)
+ * carry to the row's value (reading Z21).  Same arguments,
+ * results and tolerance as msp_spmv (empty rows get +0.0); a row split
+ * across CTAs is rounded twice (stored part, then + carries).  Async.
+ * ------------------------------------------------------------------------ */
+msp_status msp_spmv_nnz_split_workspace(const msp_csr *A, size_t *bytes);
+msp_status msp_spmv_nnz_split(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes,
+                              void *stream);
+
+/* ------------------------------------------------------------------------
  * SpAdd  C = A + B   (P:496-550 union of (row,col) tuples in Algorithm 1
  * order P:476-490; balanced path P:686-790; two phases P:816-838)
  *

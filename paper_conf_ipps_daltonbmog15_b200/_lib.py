@@ -22,7 +22,7 @@ STATUS = {0: "MSP_OK", 1: "MSP_ERR_ARG", 2: "MSP_ERR_DTYPE", 3: "MSP_ERR_SHAPE",
 # every symbol include/msp.h declares (checked by tests/test_abi.py)
 EXPORTS = [
     "msp_status_string", "msp_last_error", "msp_version", "msp_launch_count",
-    "msp_spmv_workspace", "msp_spmv",
+    "msp_spmv_workspace", "msp_spmv", "msp_spmv_nnz_split_workspace", "msp_spmv_nnz_split",
     "msp_spadd_workspace", "msp_spadd_symbolic", "msp_spadd_numeric",
     "msp_spgemm_setup_workspace", "msp_spgemm_setup", "msp_spgemm_symbolic", "msp_spgemm_numeric",
     "msp_csr_check", "msp_row_split", "msp_rebase_offsets",
@@ -63,6 +63,8 @@ _SIGS = {
     "msp_launch_count": (ctypes.c_uint64, []),
     "msp_spmv_workspace": (ctypes.c_int, [_csr_p, _P(_sz)]),
     "msp_spmv": (ctypes.c_int, [_csr_p, _vp, _vp, _vp, _sz, _vp]),
+    "msp_spmv_nnz_split_workspace": (ctypes.c_int, [_csr_p, _P(_sz)]),
+    "msp_spmv_nnz_split": (ctypes.c_int, [_csr_p, _vp, _vp, _vp, _sz, _vp]),
     "msp_spadd_workspace": (ctypes.c_int, [_csr_p, _csr_p, _P(_sz)]),
     "msp_spadd_symbolic": (ctypes.c_int, [_csr_p, _csr_p, _vp, _P(_i64), _vp, _sz, _vp]),
     "msp_spadd_numeric": (ctypes.c_int, [_csr_p, _csr_p, _vp, _vp, _vp, _vp, _sz, _vp]),

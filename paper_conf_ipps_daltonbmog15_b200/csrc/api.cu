@@ -222,6 +222,34 @@ msp_status msp_spmv(const msp_csr *A, const void *x, void *y, void *ws, size_t w
     return spmv_run(A, x, y, ws, ws_bytes, as_stream(stream));
 }
 
+msp_status msp_spmv_nnz_split_workspace(const msp_csr *A, size_t *bytes)
+{
+    clear_error();
+    msp_status st = check_csr(A, "A");
+    if (st != MSP_OK) return st;
+    if (!bytes) return MSP_ERR_ARG;
+    *bytes = spmv_nnz_ws_bytes(A) + kValidateBytes;
+    return MSP_OK;
+}
+
+msp_status msp_spmv_nnz_split(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, void *stream)
+{
+    clear_error();
+    msp_status st = check_csr(A, "A");
+    if (st != MSP_OK) return st;
+    if ((A->ncols > 0 && !x) || (A->nrows > 0 && !y) || !ws) {
+        set_error("spmv_nnz_split: NULL x, y or workspace");
+        return MSP_ERR_ARG;
+    }
+    if (ws_bytes < spmv_nnz_ws_bytes(A)) {
+        set_error("spmv_nnz_split: workspace %zu < %zu bytes", ws_bytes, spmv_nnz_ws_bytes(A));
+        return MSP_ERR_WORKSPACE;
+    }
+    st = debug_validate(A, 0, ws, ws_bytes, spmv_nnz_ws_bytes(A), as_stream(stream), "spmv_nnz_split A");
+    if (st != MSP_OK) return st;
+    return spmv_nnz_run(A, x, y, ws, ws_bytes, as_stream(stream));
+}
+
 // ------------------------------------------------------------------ SpAdd
 static msp_status check_pair_add(const msp_csr *A, const msp_csr *B)
 {

@@ -57,6 +57,8 @@ msp_status scan_i64_to_i64(const int64_t *in, int64_t *out, int64_t n, void *ws,
 // result; *overflow_dev set to 1 if the total exceeds INT32_MAX.
 msp_status scan_counts_to_offsets_i32(int32_t *counts, int64_t n, int64_t *total_dev, void *ws,
                                       size_t ws_bytes, cudaStream_t s);
+// pos[i] = number of nonempty rows before row i, i in [0, m] (row compaction)
+msp_status scan_nonempty_rows(const int32_t *rp, int64_t m, int64_t *pos, void *ws, size_t ws_bytes, cudaStream_t s);
 // S[j] = sum_{k<j} (Brp[Acol[k]+1] - Brp[Acol[k]]), j in [0, nnzA] (SpGEMM setup)
 msp_status scan_widths_to_S(const int32_t *Acol, const int32_t *Brp, int64_t nnzA, int64_t *S, void *ws,
                             size_t ws_bytes, cudaStream_t s);
@@ -66,6 +68,10 @@ size_t spmv_ws_bytes(const msp_csr *A);
 msp_status spmv_run(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s);
 // warp-tile row-aligned SpMV (spmv_wt.cu), K odd in 15..31
 msp_status spmv_wt_run(int K, const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s);
+
+// the paper's own SpMV decomposition (nnz-only split + row compaction), f4
+size_t spmv_nnz_ws_bytes(const msp_csr *A);
+msp_status spmv_nnz_run(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s);
 
 size_t spadd_ws_bytes(const msp_csr *A, const msp_csr *B);
 msp_status spadd_symbolic_run(const msp_csr *A, const msp_csr *B, int32_t *Crp, int64_t *nnzC, void *ws,

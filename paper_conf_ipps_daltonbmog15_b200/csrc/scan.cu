@@ -37,6 +37,10 @@ struct LoadWidth {  // nnz of the B row referenced by A nonzero i
         return int64_t(__ldg(brp + k + 1)) - __ldg(brp + k);
     }
 };
+struct LoadNonEmpty {  // 1 if row i has nonzeros
+    const int32_t *rp;
+    __device__ int64_t operator()(int64_t i) const { return __ldg(rp + i + 1) > __ldg(rp + i) ? 1 : 0; }
+};
 struct StoreI64 {
     int64_t *p;
     __device__ void operator()(int64_t i, int64_t v) const { p[i] = v; }
@@ -189,6 +193,11 @@ msp_status scan_counts_to_offsets_i32(int32_t *counts, int64_t n, int64_t *total
 msp_status scan_i64_to_i64(const int64_t *in, int64_t *out, int64_t n, void *ws, size_t ws_bytes, cudaStream_t s)
 {
     return run_scan<LoadI64, StoreI64, true>(LoadI64{in}, StoreI64{out}, n, nullptr, out, ws, ws_bytes, s);
+}
+
+msp_status scan_nonempty_rows(const int32_t *rp, int64_t m, int64_t *pos, void *ws, size_t ws_bytes, cudaStream_t s)
+{
+    return run_scan<LoadNonEmpty, StoreI64, true>(LoadNonEmpty{rp}, StoreI64{pos}, m, nullptr, pos, ws, ws_bytes, s);
 }
 
 msp_status scan_widths_to_S(const int32_t *Acol, const int32_t *Brp, int64_t nnzA, int64_t *S, void *ws,

@@ -933,7 +933,7 @@ int wt_choice()
     static int v = -1;
     if (v < 0) {
         const char *e = getenv("MSP_SPMV_WT");
-        v = (e && atoi(e) == 0) ? 0 : 1;
+        v = e ? atoi(e) : 1;  // 0: CTA-tile kernel, 2: warp tiles for every K (tuning)
     }
     return v;
 }
@@ -962,7 +962,7 @@ msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_
     switch (shape) {
     case -1: {
         const int K = k_choice(A);
-        if (wt_choice() && K >= 15) return spmv_wt_run(K, A, x, y, ws, ws_bytes, s);
+        if (wt_choice() && (K >= 15 || wt_choice() == 2)) return spmv_wt_run(K, A, x, y, ws, ws_bytes, s);
         return nw_choice() == 8 ? launch_k<V, 8>(K, A, x, y, ws, ws_bytes, s)
                                 : launch_k<V, 4>(K, A, x, y, ws, ws_bytes, s);
     }

@@ -77,10 +77,11 @@ struct WtCfg {
     static constexpr int THREADS = (NW + 1) * 32;        // + producer warp
     static constexpr int SLOT_BYTES = int(((4 + sizeof(V)) * T + 64 + 15) / 16 * 16);
     static constexpr int WMAP_BYTES = (32 * 4 + TI * 2 + 15) / 16 * 16;  // lane masks + row per position
-    static constexpr int RL = 128;                       // look-back ring (warp tiles)
+    static constexpr int RL = 256;                       // look-back ring (warp tiles; > STAGES*NSUB + NW)
     static constexpr int SMEM = STAGES * SLOT_BYTES + NW * WMAP_BYTES + RL * 16 + STAGES * 48 + 256;
     static_assert(K % 2 == 1 && K < 32, "K odd and < 32");
     static_assert(SMEM <= 227 * 1024, "shared memory");
+    static_assert(RL > STAGES * NSUB + 2 * NW, "look-back ring must cover the tiles in flight");
 };
 
 __device__ __forceinline__ double ldg_xv(const double *p)
@@ -494,7 +495,7 @@ msp_status launch_wt(const msp_csr *A, const void *x, void *y, void *ws, size_t 
     // 168 registers per thread (each sub-partition holds 16K registers);
     // 3 stages of up to 8 warp tiles (about 62 KB each)
     constexpr int NSUB0 = (188 * 1024 / 3) / int((4 + sizeof(V)) * 32 * K);
-    using C = WtCfg<V, K, 11, (NSUB0 < 8 ? NSUB0 : 8), 3>;
+    using C = WtCfg<V, K, 11, (NSUB0 < 24 ? NSUB0 : 24), 3>;
     auto kern = spmv_wt_kernel<V, C>;
     int occ = 1;
     msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), C::SMEM, "spmv_wt: smem", C::THREADS, &occ);
@@ -532,6 +533,8 @@ msp_status spmv_wt_run(int K, const msp_csr *A, const void *x, void *y, void *ws
 {
     const bool f64 = A->dtype == MSP_F64;
     switch (K) {
+    case 7: return f64 ? launch_wt<double, 7>(A, x, y, ws, ws_bytes, s) : launch_wt<float, 7>(A, x, y, ws, ws_bytes, s);
+    case 11: return f64 ? launch_wt<double, 11>(A, x, y, ws, ws_bytes, s) : launch_wt<float, 11>(A, x, y, ws, ws_bytes, s);
     case 15: return f64 ? launch_wt<double, 15>(A, x, y, ws, ws_bytes, s) : launch_wt<float, 15>(A, x, y, ws, ws_bytes, s);
     case 19: return f64 ? launch_wt<double, 19>(A, x, y, ws, ws_bytes, s) : launch_wt<float, 19>(A, x, y, ws, ws_bytes, s);
     case 23: return f64 ? launch_wt<double, 23>(A, x, y, ws, ws_bytes, s) : launch_wt<float, 23>(A, x, y, ws, ws_bytes, s);

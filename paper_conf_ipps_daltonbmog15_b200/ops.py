@@ -124,6 +124,21 @@ def spmv(A: CsrTensor, x: torch.Tensor, out: torch.Tensor | None = None, stream=
     return y
 
 
+def spmv_nnz_split(A: CsrTensor, x: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+    """y = A x with the paper's own decomposition (nnz-only split + row
+    compaction): the f4(i) ablation of spmv()."""
+    if x.dtype != A.dtype or x.device != A.device or x.numel() != A.shape[1] or not x.is_contiguous():
+        raise ValueError("x must be a contiguous vector of A.dtype on A.device with A.shape[1] entries")
+    y = out if out is not None else torch.empty(A.shape[0], dtype=A.dtype, device=A.device)
+    a = A.c()
+    n = ctypes.c_size_t(0)
+    check("msp_spmv_nnz_split_workspace", lib().msp_spmv_nnz_split_workspace(ctypes.byref(a), ctypes.byref(n)))
+    ws = workspace(int(n.value), A.device, "spmv_nnz", stream)
+    check("msp_spmv_nnz_split", lib().msp_spmv_nnz_split(ctypes.byref(a), x.data_ptr(), y.data_ptr(), ws.data_ptr(),
+                                                         ws.numel(), _stream_ptr(A.device, stream)))
+    return y
+
+
 # ----------------------------------------------------------------- SpAdd
 
 class SpAddPlan:
