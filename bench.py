@@ -401,7 +401,23 @@ def table_configs(msp, torch, dev, names, peak, flush):
             ms = float(np.mean([a.elapsed_time(b) for a, b in ts]))
             by = spmv_alg_bytes(A.m, A.n, A.nnz, vs)
             ent["spmv"] = {"ms": ms, "alg_bytes": by, "GB_s": by / ms / 1e6, "frac_hbm": by / ms / 1e6 / peak,
-                           "GFLOP_s": 2 * A.nnz / ms / 1e6, "l2": "flushed" if small else "inputs > L2"}
+                           "GFLOP_s": 2 * A.nnz / ms / 1e6, "l2": "flushed" if small else "inputs > L2",
+                           "kernel": spmv_kernel_name(A.m, A.nnz)}
+            # f4(i) ablation: the paper's nnz-only split with row compaction
+            for _ in range(2):
+                msp.spmv_nnz_split(dA, x, out=y)
+            ts = []
+            for _ in range(reps):
+                if small:
+                    flush()
+                a = tm.ev()
+                msp.spmv_nnz_split(dA, x, out=y)
+                b = tm.ev()
+                ts.append((a, b))
+            torch.cuda.synchronize(dev)
+            ms2 = float(np.mean([a.elapsed_time(b) for a, b in ts]))
+            ent["spmv_nnz_split"] = {"ms": ms2, "GB_s": by / ms2 / 1e6, "frac_hbm": by / ms2 / 1e6 / peak,
+                                     "vs_merge_grid": ms / ms2}
             del x, y
         if "spadd" in BJ_OPS[name]:
             T = transposed(name)

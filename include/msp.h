@@ -269,6 +269,13 @@ msp_status msp_row_split(const int32_t *row_offsets_host, int32_t nrows, int32_t
 msp_status msp_rebase_offsets(const int32_t *in, int32_t *out, int64_t n, int64_t base,
                               void *stream);
 
+/* Gather dst[i] = src[idx[i]], i in [0, n), of value_bytes (4 or 8) each:
+ * packs the halo values a rank sends to its neighbours in the distributed
+ * SpMV without full-x replication.
+ * Device pointers; idx entries must be valid indices of src.  Async. */
+msp_status msp_gather_values(const void *src, const int32_t *idx, int64_t n, int32_t value_bytes, void *dst,
+                             void *stream);
+
 #ifdef __cplusplus
 }
 #endif

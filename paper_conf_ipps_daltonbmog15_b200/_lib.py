@@ -25,7 +25,7 @@ EXPORTS = [
     "msp_spmv_workspace", "msp_spmv", "msp_spmv_nnz_split_workspace", "msp_spmv_nnz_split",
     "msp_spadd_workspace", "msp_spadd_symbolic", "msp_spadd_numeric",
     "msp_spgemm_setup_workspace", "msp_spgemm_setup", "msp_spgemm_symbolic", "msp_spgemm_numeric",
-    "msp_csr_check", "msp_row_split", "msp_rebase_offsets",
+    "msp_csr_check", "msp_row_split", "msp_rebase_offsets", "msp_gather_values",
     "msp_set_op_workspace", "msp_set_operation",
 ]
 
@@ -77,6 +77,7 @@ _SIGS = {
     "msp_csr_check": (ctypes.c_int, [_csr_p, ctypes.c_int, _P(_i32), _vp, _sz, _vp]),
     "msp_row_split": (ctypes.c_int, [_vp, _i32, _i32, _vp]),
     "msp_rebase_offsets": (ctypes.c_int, [_vp, _vp, _i64, _i64, _vp]),
+    "msp_gather_values": (ctypes.c_int, [_vp, _vp, _i64, _i32, _vp, _vp]),
     "msp_set_op_workspace": (ctypes.c_int, [_i64, _i64, _P(_sz)]),
     "msp_set_operation": (ctypes.c_int, [ctypes.c_int, _vp, _vp, _i64, _vp, _vp, _i64, _i32, _i32, _vp, _vp, _i64,
                                           _P(_i64), _vp, _sz, _vp]),

@@ -413,6 +413,18 @@ msp_status msp_rebase_offsets(const int32_t *in, int32_t *out, int64_t n, int64_
     return rebase_run(in, out, n, base, as_stream(stream));
 }
 
+msp_status msp_gather_values(const void *src, const int32_t *idx, int64_t n, int32_t value_bytes, void *dst,
+                             void *stream)
+{
+    clear_error();
+    if (n < 0 || (n > 0 && (!src || !idx || !dst))) return MSP_ERR_ARG;
+    if (value_bytes != 4 && value_bytes != 8) {
+        set_error("gather: value_bytes must be 4 or 8");
+        return MSP_ERR_DTYPE;
+    }
+    return gather_run(src, idx, n, value_bytes, dst, as_stream(stream));
+}
+
 msp_status msp_set_op_workspace(int64_t nA, int64_t nB, size_t *bytes)
 {
     clear_error();

@@ -2,6 +2,8 @@
 // "sorted by row and row-wise internally sorted by column" precondition of
 // the union formulation) and a row-offset rebase helper used for
 // multi-GPU row-block views.
+#include <algorithm>
+
 #include "common.cuh"
 #include "internal.h"
 
@@ -76,6 +78,35 @@ msp_status rebase_run(const int32_t *in, int32_t *out, int64_t n, int64_t base, 
     if (blocks > 148 * 16) blocks = 148 * 16;
     rebase_kernel<<<unsigned(blocks), 256, 0, s>>>(in, out, n, base);
     return last_launch("rebase_kernel");
+}
+
+}  // namespace msp
+
+// ---------------------------------------------------------------- gather
+namespace msp {
+namespace {
+
+template <typename T>
+__global__ void gather_kernel(const T *__restrict__ src, const int32_t *__restrict__ idx, int64_t n,
+                              T *__restrict__ dst)
+{
+    for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
+        dst[i] = src[idx[i]];
+}
+
+}  // namespace
+
+msp_status gather_run(const void *src, const int32_t *idx, int64_t n, int value_bytes, void *dst, cudaStream_t s)
+{
+    if (n <= 0) return MSP_OK;
+    const unsigned blocks = unsigned(std::min<int64_t>(ceil_div(n, 256), 148 * 16));
+    if (value_bytes == 8)
+        gather_kernel<uint64_t><<<blocks, 256, 0, s>>>(static_cast<const uint64_t *>(src), idx, n,
+                                                       static_cast<uint64_t *>(dst));
+    else
+        gather_kernel<uint32_t><<<blocks, 256, 0, s>>>(static_cast<const uint32_t *>(src), idx, n,
+                                                       static_cast<uint32_t *>(dst));
+    return last_launch("gather_kernel");
 }
 
 }  // namespace msp

@@ -94,6 +94,7 @@ size_t set_op_ws_bytes(int64_t na, int64_t nb);
 msp_status set_op_run(int op, const void *A, const void *Av, int64_t na, const void *B, const void *Bv, int64_t nb,
                       int key_bytes, int val_bytes, void *C, void *Cv, int64_t cap, int64_t *nC_host, void *ws,
                       size_t ws_bytes, cudaStream_t s);
+msp_status gather_run(const void *src, const int32_t *idx, int64_t n, int value_bytes, void *dst, cudaStream_t s);
 msp_status rebase_run(const int32_t *in, int32_t *out, int64_t n, int64_t base, cudaStream_t s);
 
 }  // namespace msp

@@ -78,7 +78,7 @@ struct WtCfg {
     static constexpr int SLOT_BYTES = int(((4 + sizeof(V)) * T + 64 + 15) / 16 * 16);
     static constexpr int WMAP_BYTES = (32 * 4 + TI * 2 + 15) / 16 * 16;  // lane masks + row per position
     static constexpr int RL = 256;                       // look-back ring (warp tiles; > STAGES*NSUB + NW)
-    static constexpr int SMEM = STAGES * SLOT_BYTES + NW * WMAP_BYTES + RL * 16 + STAGES * 48 + 256;
+    static constexpr int SMEM = STAGES * SLOT_BYTES + NW * WMAP_BYTES + RL * 32 + STAGES * 48 + 256;
     static_assert(K % 2 == 1 && K < 32, "K odd and < 32");
     static_assert(SMEM <= 227 * 1024, "shared memory");
     static_assert(RL > STAGES * NSUB + 2 * NW, "look-back ring must cover the tiles in flight");
@@ -156,22 +156,41 @@ __device__ __forceinline__ int stage_split(const int32_t *rpb, int j_s, int d, i
     return lo + __popc(__ballot_sync(0xffffffffu, pred));
 }
 
-// look-back record of a tile: value and a tag word (tile+1) << 2 | kind,
-// kind 1 = aggregate (flag bit 0 of `f`), 2 = inclusive carry-out
+// Look-back record of a tile.  The aggregate (trailing sum) and the
+// inclusive carry-out live in SEPARATE fields, each written once before its
+// bit in the tag word ((tile+1) << 2 | 1 aggregate | 2 inclusive): a reader
+// that sees bit 1 only must never read an inclusive value written after it
+// checked the tag (an earlier single-value record was upgraded in place and
+// could be read half-way: nondeterministic double counting on long rows).
 struct alignas(16) LbRec {
-    double v;
-    int f;
+    double agg;   // trailing sum of the tile
+    double inc;   // inclusive carry-out (the carry into the next tile)
+    int f_agg;    // the tile has a row end
+    int f_inc;    // some tile of the CTA up to this one has a row end
     int tag;
+    int pad;
 };
 
-__device__ __forceinline__ void lb_publish(LbRec *r, double v, int f, int tag)
+__device__ __forceinline__ void lb_publish_agg(LbRec *r, double v, int tile)
 {
-    // value first, then the tag with release semantics inside the CTA
-    *reinterpret_cast<volatile double *>(&r->v) = v;
-    *reinterpret_cast<volatile int *>(&r->f) = f;
+    *reinterpret_cast<volatile double *>(&r->agg) = v;
+    *reinterpret_cast<volatile int *>(&r->f_agg) = 0;
     __threadfence_block();
-    *reinterpret_cast<volatile int *>(&r->tag) = tag;
+    *reinterpret_cast<volatile int *>(&r->tag) = ((tile + 1) << 2) | 1;
 }
+
+__device__ __forceinline__ void lb_publish_inc(LbRec *r, double agg, double inc, int f_agg, int f_inc, int tile)
+{
+    *reinterpret_cast<volatile double *>(&r->agg) = agg;
+    *reinterpret_cast<volatile double *>(&r->inc) = inc;
+    *reinterpret_cast<volatile int *>(&r->f_agg) = f_agg;
+    *reinterpret_cast<volatile int *>(&r->f_inc) = f_inc;
+    __threadfence_block();
+    *reinterpret_cast<volatile int *>(&r->tag) = ((tile + 1) << 2) | 3;
+}
+
+// (the aggregate fields of a record are rewritten with the same values when
+// its inclusive carry is published, so a concurrent aggregate read is exact)
 
 template <typename V, class C>
 __global__ void __launch_bounds__(C::THREADS, 1)
@@ -285,17 +304,12 @@ spmv_wt_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const int
                 int tg;
                 while (((tg = *reinterpret_cast<volatile int *>(&rec->tag)) >> 2) != j + 1) {}
                 __threadfence_block();
-                const double v = *reinterpret_cast<volatile double *>(&rec->v);
-                if ((tg & 3) == 2) {  // inclusive: carry-out of tile j, head status in f
-                    c = v + c;
-                    head = *reinterpret_cast<volatile int *>(&rec->f) == 0;
+                if (tg & 2) {  // inclusive carry-out of tile j, head status in f_inc
+                    c = *reinterpret_cast<volatile double *>(&rec->inc) + c;
+                    head = *reinterpret_cast<volatile int *>(&rec->f_inc) == 0;
                     break;
                 }
-                c = v + c;
-                if (*reinterpret_cast<volatile int *>(&rec->f)) {
-                    head = false;
-                    break;
-                }
+                c = *reinterpret_cast<volatile double *>(&rec->agg) + c;  // aggregate of a tile without row ends
             }
             if (has_rows) {
                 const double v = v0 + c;
@@ -305,9 +319,9 @@ spmv_wt_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const int
                     s_head_val = v;
                 }
             } else {
-                // no row end in tile tt: publish its inclusive carry-out (f = 1
-                // if some earlier tile of the CTA had a row end)
-                lb_publish(&lb[tt & (RL - 1)], c + agg, head ? 0 : 1, ((tt + 1) << 2) | 2);
+                // no row end in tile tt: publish its inclusive carry-out (f_inc
+                // = 1 if some earlier tile of the CTA had a row end)
+                lb_publish_inc(&lb[tt & (RL - 1)], agg, c + agg, 0, head ? 0 : 1, tt);
             }
         };
         for (int t = warp; t < ntiles; t += NW) {
@@ -376,6 +390,15 @@ spmv_wt_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const int
             }
             __syncwarp();
             const unsigned mask = wmask[lane];
+#ifndef MSP_WT_NO_VV_FENCE
+            {   // the values must be IN registers before the slot is handed back
+                // to the TMA engine: consume every vv register (scoreboard wait)
+                unsigned long long acc = 0;
+#pragma unroll
+                for (int u = 0; u < K; ++u) acc |= __double_as_longlong(vv[u]);
+                asm volatile("" ::"l"(acc));
+            }
+#endif
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[slot]);  // this warp tile of the stage is in regs / the map
             if (lane == 0) WTR(t, 4);  // released
@@ -422,8 +445,8 @@ spmv_wt_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const int
                 if (lane == flane) nv = v;
                 else y[first_r] = V(v);
             }
-            if (lane == 0 && fmask) lb_publish(&lb[t & (RL - 1)], agg, 1, ((t + 1) << 2) | 2);  // carry-out known
-            else if (lane == 0) lb_publish(&lb[t & (RL - 1)], agg, 0, ((t + 1) << 2) | 1);     // aggregate only
+            if (lane == 0 && fmask) lb_publish_inc(&lb[t & (RL - 1)], agg, agg, 1, 1, t);  // carry-out known
+            else if (lane == 0) lb_publish_agg(&lb[t & (RL - 1)], agg, t);                  // aggregate only
             // ---- finish the previous tile of this warp (deferred look-back) ----
             if (pend_t >= 0) {
                 const int hr = __shfl_sync(0xffffffffu, pend_r, pend_fl >= 0 ? pend_fl : 0);
@@ -450,9 +473,9 @@ spmv_wt_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const int
         const int j = ntiles - 1;
         LbRec *rec = &lb[j & (RL - 1)];
         int tg;
-        while (((tg = *reinterpret_cast<volatile int *>(&rec->tag)) >> 2) != j + 1 || (tg & 3) != 2) {}
+        while (((tg = *reinterpret_cast<volatile int *>(&rec->tag)) >> 2) != j + 1 || !(tg & 2)) {}
         __threadfence_block();
-        s_carry_val = *reinterpret_cast<volatile double *>(&rec->v);
+        s_carry_val = *reinterpret_cast<volatile double *>(&rec->inc);
     }
     __syncthreads();
     if (tid == 0) {

@@ -16,6 +16,8 @@ NVLink/NVSwitch on GPUs; gloo in the CPU tests of the exchange logic).
   replicated C is wanted (C may instead stay distributed by row blocks).
 * `block_view` / `concat_blocks` are the zero-copy row-block views and the
   concatenation used on one device (the P-block parity tests).
+* `HaloSpmv`: SpMV without replicating x -- a one-time halo plan and one
+  all_to_all of the halo values per SpMV.
 
 Compute happens in libmsp kernels (CUDA tensors); only data movement and
 offset rebasing are done here.  CPU tensors are accepted so that the exchange
@@ -182,3 +184,89 @@ def dist_spgemm(A_blk: CsrTensor, B_blk: CsrTensor, group=None, gather_c: bool =
     plan.symbolic()
     C_blk = plan.numeric()
     return gather_csr_blocks(C_blk, group) if gather_c else C_blk
+
+
+class HaloSpmv:
+    """Distributed SpMV WITHOUT replicating x: a halo
+    exchange instead of the all-gather.
+
+    x is owned in equal slices of ceil(n/P) entries (as for `allgather_x`).
+    Setup (host, once per matrix): the rank's row block lists the columns it
+    references; those owned by other ranks form its halo, sorted by global
+    index -- hence grouped by owner rank.  The per-owner request lists are
+    exchanged once (all_to_all), so every rank knows which of its x entries
+    each neighbour needs; the block's column indices are renumbered into a
+    local x = [own slice | halo from rank 0 | halo from rank 1 | ...].
+    Per SpMV: the rank packs the values its neighbours need
+    (`msp_gather_values`), ONE all_to_all_single delivers every halo
+    straight into the local x, and the local SpMV (libmsp) runs on the
+    renumbered block.  For a banded / stencil matrix the halo is a few planes
+    (C2 slabs: 2 x 10^4 entries per neighbour) instead of the whole x; for
+    uniformly random columns (C5) it approaches the all-gather.
+    """
+
+    def __init__(self, rp_blk, col_blk, val_blk, n: int, group=None, device=None):
+        import numpy as np
+        self.group = group
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        P, r = self.world, self.rank
+        self.n = n
+        self.ns = -(-n // P)
+        own0 = r * self.ns
+        self.own_len = max(0, min(n, own0 + self.ns) - own0)
+        cols = np.asarray(col_blk, dtype=np.int64)
+        uniq = np.unique(cols)
+        owner = uniq // self.ns
+        remote = uniq[owner != r]
+        rown = remote // self.ns
+        need = np.bincount(rown, minlength=P).astype(np.int64)  # entries this rank needs from each owner
+        dev = device if device is not None else torch.device("cpu")
+        cpu = not (isinstance(dev, torch.device) and dev.type == "cuda") and not (isinstance(dev, str) and
+                                                                                   dev.startswith("cuda"))
+        coll_dev = torch.device("cpu") if cpu else torch.device(dev)
+        # exchange request counts, then the request lists (global indices)
+        need_t = torch.as_tensor(need, device=coll_dev)
+        give_t = torch.empty_like(need_t)
+        dist.all_to_all_single(give_t, need_t, group=group)
+        give = give_t.cpu().numpy().astype(np.int64)  # entries each rank needs from this rank
+        req = torch.as_tensor(remote.astype(np.int64), device=coll_dev)
+        got = torch.empty(int(give.sum()), dtype=torch.int64, device=coll_dev)
+        dist.all_to_all_single(got, req, output_split_sizes=give.tolist(), input_split_sizes=need.tolist(),
+                               group=group)
+        send_idx = (got.cpu().numpy() - own0).astype(np.int32)  # positions in this rank's slice
+        assert send_idx.size == 0 or (send_idx.min() >= 0 and send_idx.max() < self.own_len)
+        self.send_counts, self.recv_counts = give.tolist(), need.tolist()
+        self.halo_len = int(remote.size)
+        # renumbered columns: own -> c - own0, remote -> own_len + rank in `remote`
+        mine = (cols // self.ns) == r
+        local = np.empty(cols.size, dtype=np.int64)
+        local[mine] = cols[mine] - own0
+        local[~mine] = self.own_len + np.searchsorted(remote, cols[~mine])
+        m_blk = len(rp_blk) - 1
+        self.A = CsrTensor.from_arrays(np.asarray(rp_blk, dtype=np.int32), local.astype(np.int32), val_blk,
+                                       (m_blk, self.own_len + self.halo_len), dev)
+        self.send_idx = torch.as_tensor(send_idx, device=dev)
+        self.x_local = torch.zeros(self.own_len + self.halo_len, dtype=self.A.val.dtype, device=dev)
+        self.send_buf = torch.empty(int(send_idx.size), dtype=self.A.val.dtype, device=dev)
+
+    @property
+    def x_own(self) -> torch.Tensor:
+        """This rank's slice of x (write the vector here before `spmv`)."""
+        return self.x_local[:self.own_len]
+
+    def exchange(self):
+        """Halo values of x into x_local (pack + one all_to_all_single)."""
+        if self.send_buf.is_cuda:
+            from .ops import gather_values
+            gather_values(self.x_own, self.send_idx, out=self.send_buf)
+        else:  # host plumbing for the gloo tests
+            self.send_buf.copy_(self.x_own[self.send_idx.long()])
+        dist.all_to_all_single(self.x_local[self.own_len:], self.send_buf, output_split_sizes=self.recv_counts,
+                               input_split_sizes=self.send_counts, group=self.group)
+
+    def spmv(self, out: torch.Tensor | None = None) -> torch.Tensor:
+        """y rows of this rank = A_blk @ x (halo exchange, then libmsp SpMV)."""
+        from .ops import spmv
+        self.exchange()
+        return spmv(self.A, self.x_local, out=out)

@@ -301,6 +301,17 @@ def rebase_offsets(rp: torch.Tensor, base: int, out: torch.Tensor | None = None)
     return out
 
 
+def gather_values(src: torch.Tensor, idx: torch.Tensor, out: torch.Tensor | None = None) -> torch.Tensor:
+    """out[i] = src[idx[i]] on the device (msp_gather_values; halo packing)."""
+    if idx.dtype != torch.int32 or not idx.is_contiguous() or not src.is_contiguous():
+        raise ValueError("idx int32 and contiguous tensors required")
+    out = out if out is not None else torch.empty(idx.numel(), dtype=src.dtype, device=src.device)
+    check("msp_gather_values", lib().msp_gather_values(src.data_ptr(), idx.data_ptr(), idx.numel(),
+                                                       src.element_size(), out.data_ptr(),
+                                                       _stream_ptr(src.device)))
+    return out
+
+
 # ----------------------------------------------------------------- set operations
 
 SET_OPS = {"union": 0, "intersection": 1, "difference": 2, "symmetric_difference": 3}

@@ -89,3 +89,26 @@ def test_row_blocks_one_gpu(cfg, scale, P):
         assert np.array_equal(rp, W.rp), f"{cfg} P={P} {split}: row_offsets"
         assert np.array_equal(col, W.col), f"{cfg} P={P} {split}: col_idx"
         assert np.array_equal(val, W.val), f"{cfg} P={P} {split}: values"
+
+
+def test_gather_values():
+    from paper_conf_ipps_daltonbmog15_b200 import gather_values
+    src = torch.arange(1000, dtype=torch.float64, device="cuda") * 1.5
+    idx = torch.as_tensor(np.random.default_rng(1).integers(0, 1000, 777), dtype=torch.int32, device="cuda")
+    assert torch.equal(gather_values(src, idx), src[idx.long()])
+    s32 = torch.arange(100, dtype=torch.float32, device="cuda")
+    i32 = torch.tensor([5, 0, 99], dtype=torch.int32, device="cuda")
+    assert gather_values(s32, i32).tolist() == [5.0, 0.0, 99.0]
+
+
+def test_halo_spmv_world1(pg):
+    """The halo-exchange SpMV on one rank (NCCL): no halo, renumbered columns
+    equal the originals, result equals the oracle bit for bit (int mode)."""
+    from paper_conf_ipps_daltonbmog15_b200 import dist as mdist
+    A = gen.config("C4", "int", scale=0.02)
+    x = gen.x_vector(A.n, "int")
+    plan = mdist.HaloSpmv(A.rp, A.col, A.val, A.n, device=torch.device("cuda", 0))
+    assert plan.halo_len == 0 and plan.own_len == A.n
+    plan.x_own.copy_(torch.as_tensor(x, device="cuda"))
+    y = plan.spmv().cpu().numpy()
+    assert np.array_equal(y, oracle.spmv(A, x)[0])

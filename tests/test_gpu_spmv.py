@@ -142,3 +142,27 @@ def test_cta_boundary_before_row_end(L):
         x = gen.x_vector(n, "int")
         y = run(A, x)
         assert np.array_equal(y, oracle.spmv(A, x)[0]), f"m={m} L={L}"
+
+
+def test_warp_tiles_long_rows():
+    """The warp-tile kernel (chosen when the mean row length is >= 20) on rows
+    that span many warp tiles and CTAs next to stencil-length rows and empty
+    rows: the decoupled look-back over tiles without row ends must give the
+    exact result, run to run (a record upgraded in place once let a reader
+    take an inclusive carry for an aggregate)."""
+    rng = np.random.default_rng(11)
+    for i, lens in enumerate([[27] * 5000 + [200_000] + [27] * 5000,
+                              [300_000] + list(rng.choice([0, 27, 27, 27, 3000], 20_000)),
+                              list(rng.integers(0, 3000, 400))]):
+        n = 400_000
+        g = np.random.default_rng(20 + i)
+        cols = [np.unique(g.integers(0, n, int(L) + int(L) // 8 + 4))[:int(L)] for L in lens]
+        lens = [c.size for c in cols]
+        rp = np.concatenate([[0], np.cumsum(lens)]).astype(np.int32)
+        col = np.concatenate(cols).astype(np.int32)
+        A = gen.CSR(len(lens), n, rp, col, gen.int_values(col.size, 30 + i))
+        assert A.nnz >= 20 * A.m  # the warp-tile path
+        x = gen.x_vector(A.n, "int")
+        want = oracle.spmv(A, x)[0]
+        for _ in range(3):
+            assert np.array_equal(run(A, x), want), f"case {i}"
