@@ -209,6 +209,33 @@ msp_status msp_spgemm_numeric(const msp_csr *A, const msp_csr *B, const void *se
                               int32_t *C_col_idx, void *C_vals, void *stream);
 
 /* ------------------------------------------------------------------------
+ * SpGEMM with the paper's own sort pipeline (ablation, SURVEY §8(f) f2;
+ * P:994-1212, Figs 3-4).  After msp_spgemm_setup (same setup_ws / info):
+ * symbolic = phase 1 (per tile of 2048 products: expand (row, col), one
+ * keys-only radix sort on the ceil(log2 n) column bits with the tile index
+ * in the low bits, duplicates adjacent, 16-bit permutation + head flags
+ * stored, reduced entries compacted in tile order) and phase 2 (a global
+ * LSD radix sort of the reduced (row, col) keys that only computes their
+ * permutation), then C.row_offsets and *nnz_C (synchronises twice).
+ * Numeric = phase 3 (re-expansion with values, each tile's stored
+ * permutation, reduction by the stored duplicate flags, values stored at
+ * their sorted positions) and a global reduce-by-key into C (async).  Same
+ * results as msp_spgemm_* (structure bit-exact, values within tolerance,
+ * deterministic); Nprods must be < 2^32.  ws: msp_spgemm_radix_workspace()
+ * bytes, untouched between symbolic and numeric.
+ * ------------------------------------------------------------------------ */
+msp_status msp_spgemm_radix_workspace(const msp_csr *A, const msp_csr *B, const msp_spgemm_info *info_host,
+                                      size_t *bytes);
+msp_status msp_spgemm_radix_symbolic(const msp_csr *A, const msp_csr *B, const void *setup_ws,
+                                     size_t setup_ws_bytes, void *ws, size_t ws_bytes,
+                                     const msp_spgemm_info *info_host, int32_t *C_row_offsets,
+                                     int64_t *nnzC_host, void *stream);
+msp_status msp_spgemm_radix_numeric(const msp_csr *A, const msp_csr *B, const void *setup_ws,
+                                    size_t setup_ws_bytes, void *ws, size_t ws_bytes,
+                                    const msp_spgemm_info *info_host, const int32_t *C_row_offsets,
+                                    int32_t *C_col_idx, void *C_vals, void *stream);
+
+/* ------------------------------------------------------------------------
  * Input validation (the CSR contract of P:316-322).
  * flags_host receives a bit set: 1 = row_offsets not monotone or
  * row_offsets[0] != 0 or row_offsets[nrows] != nnz, 2 = column out of

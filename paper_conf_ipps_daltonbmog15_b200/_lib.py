@@ -25,6 +25,7 @@ EXPORTS = [
     "msp_spmv_workspace", "msp_spmv", "msp_spmv_nnz_split_workspace", "msp_spmv_nnz_split",
     "msp_spadd_workspace", "msp_spadd_symbolic", "msp_spadd_numeric",
     "msp_spgemm_setup_workspace", "msp_spgemm_setup", "msp_spgemm_symbolic", "msp_spgemm_numeric",
+    "msp_spgemm_radix_workspace", "msp_spgemm_radix_symbolic", "msp_spgemm_radix_numeric",
     "msp_csr_check", "msp_row_split", "msp_rebase_offsets", "msp_gather_values",
     "msp_set_op_workspace", "msp_set_operation",
 ]
@@ -74,6 +75,11 @@ _SIGS = {
                                            _vp]),
     "msp_spgemm_numeric": (ctypes.c_int, [_csr_p, _csr_p, _vp, _sz, _vp, _sz, _P(msp_spgemm_info), _vp, _vp, _vp,
                                           _vp]),
+    "msp_spgemm_radix_workspace": (ctypes.c_int, [_csr_p, _csr_p, _P(msp_spgemm_info), _P(_sz)]),
+    "msp_spgemm_radix_symbolic": (ctypes.c_int, [_csr_p, _csr_p, _vp, _sz, _vp, _sz, _P(msp_spgemm_info), _vp,
+                                                 _P(_i64), _vp]),
+    "msp_spgemm_radix_numeric": (ctypes.c_int, [_csr_p, _csr_p, _vp, _sz, _vp, _sz, _P(msp_spgemm_info), _vp, _vp,
+                                                _vp, _vp]),
     "msp_csr_check": (ctypes.c_int, [_csr_p, ctypes.c_int, _P(_i32), _vp, _sz, _vp]),
     "msp_row_split": (ctypes.c_int, [_vp, _i32, _i32, _vp]),
     "msp_rebase_offsets": (ctypes.c_int, [_vp, _vp, _i64, _i64, _vp]),

@@ -370,6 +370,47 @@ msp_status msp_spgemm_numeric(const msp_csr *A, const msp_csr *B, const void *se
                               C_col_idx, C_vals, as_stream(stream));
 }
 
+msp_status msp_spgemm_radix_workspace(const msp_csr *A, const msp_csr *B, const msp_spgemm_info *info_host,
+                                      size_t *bytes)
+{
+    clear_error();
+    msp_status st = check_pair_mul(A, B);
+    if (st != MSP_OK) return st;
+    if (!info_host || !bytes) return MSP_ERR_ARG;
+    *bytes = spgemm_radix_ws_bytes(A, B, info_host->nprods);
+    return MSP_OK;
+}
+
+msp_status msp_spgemm_radix_symbolic(const msp_csr *A, const msp_csr *B, const void *setup_ws, size_t setup_ws_bytes,
+                                     void *ws, size_t ws_bytes, const msp_spgemm_info *info_host,
+                                     int32_t *C_row_offsets, int64_t *nnzC_host, void *stream)
+{
+    clear_error();
+    msp_status st = check_pair_mul(A, B);
+    if (st != MSP_OK) return st;
+    if (!setup_ws || !ws || !info_host || !C_row_offsets || !nnzC_host) return MSP_ERR_ARG;
+    if (info_host->nprods >= (int64_t(1) << 32)) {
+        set_error("spgemm_radix: Nprods >= 2^32 (32-bit reduced-entry indices)");
+        return MSP_ERR_OVERFLOW;
+    }
+    if (ws_bytes < spgemm_radix_ws_bytes(A, B, info_host->nprods)) return MSP_ERR_WORKSPACE;
+    return spgemm_radix_symbolic_run(A, B, setup_ws, setup_ws_bytes, ws, ws_bytes, info_host->nprods, C_row_offsets,
+                                     nnzC_host, as_stream(stream));
+}
+
+msp_status msp_spgemm_radix_numeric(const msp_csr *A, const msp_csr *B, const void *setup_ws, size_t setup_ws_bytes,
+                                    void *ws, size_t ws_bytes, const msp_spgemm_info *info_host,
+                                    const int32_t *C_row_offsets, int32_t *C_col_idx, void *C_vals, void *stream)
+{
+    clear_error();
+    msp_status st = check_pair_mul(A, B);
+    if (st != MSP_OK) return st;
+    if (!setup_ws || !ws || !info_host || !C_row_offsets) return MSP_ERR_ARG;
+    if (ws_bytes < spgemm_radix_ws_bytes(A, B, info_host->nprods)) return MSP_ERR_WORKSPACE;
+    return spgemm_radix_numeric_run(A, B, setup_ws, setup_ws_bytes, ws, ws_bytes, info_host->nprods, C_row_offsets,
+                                    C_col_idx, C_vals, as_stream(stream));
+}
+
 // ------------------------------------------------------------------ misc
 msp_status msp_csr_check(const msp_csr *A, int require_sorted_unique, int32_t *flags_host, void *ws,
                          size_t ws_bytes, void *stream)

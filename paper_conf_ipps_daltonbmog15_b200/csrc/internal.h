@@ -88,6 +88,16 @@ msp_status spgemm_numeric_run(const msp_csr *A, const msp_csr *B, const void *ws
                               size_t b2, const msp_spgemm_info *info, const int32_t *Crp, int32_t *Ccol, void *Cval,
                               cudaStream_t s);
 
+// COO rows of A's nonzeros and the product prefix S (both in setup_ws)
+msp_status spgemm_setup_arrays(const msp_csr *A, const void *ws1, size_t b1, const int32_t **arow, const int64_t **S);
+// the paper's own SpGEMM sort pipeline (spgemm_radix.cu)
+size_t spgemm_radix_ws_bytes(const msp_csr *A, const msp_csr *B, int64_t nprods);
+msp_status spgemm_radix_symbolic_run(const msp_csr *A, const msp_csr *B, const void *ws1, size_t b1, void *ws,
+                                     size_t bytes, int64_t nprods, int32_t *Crp, int64_t *nnzC, cudaStream_t s);
+msp_status spgemm_radix_numeric_run(const msp_csr *A, const msp_csr *B, const void *ws1, size_t b1, void *ws,
+                                    size_t bytes, int64_t nprods, const int32_t *Crp, int32_t *Ccol, void *Cval,
+                                    cudaStream_t s);
+
 msp_status csr_check_run(const msp_csr *A, int sorted_unique, int32_t *flags_host, void *ws, size_t ws_bytes,
                          cudaStream_t s);
 size_t set_op_ws_bytes(int64_t na, int64_t nb);

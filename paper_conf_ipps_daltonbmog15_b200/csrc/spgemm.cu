@@ -934,6 +934,16 @@ HostInfo host_info(const msp_spgemm_info *info)
 
 }  // namespace
 
+msp_status spgemm_setup_arrays(const msp_csr *A, const void *ws1, size_t b1, const int32_t **arow, const int64_t **S)
+{
+    bool ok;
+    const SetupWs w = carve_setup(A, const_cast<void *>(ws1), b1, &ok);
+    if (!ok) return MSP_ERR_WORKSPACE;
+    *arow = w.arow;
+    *S = w.S;
+    return MSP_OK;
+}
+
 size_t spgemm_setup_ws_bytes(const msp_csr *A, const msp_csr *)
 {
     bool ok;

@@ -263,6 +263,43 @@ class SpGemmPlan:
         return CsrTensor(self.rp, col, val, (self.A.shape[0], self.B.shape[1]))
 
 
+class SpGemmRadixPlan(SpGemmPlan):
+    """SpGEMM with the paper's own sort pipeline (the f2
+    ablation): setup() as SpGemmPlan, then radix symbolic / numeric."""
+
+    def symbolic(self) -> int:
+        if self.info is None or not _owns(self.token, self.A.device, self._SLOTS[:1], self.stream):
+            self.setup()
+        n = ctypes.c_size_t(0)
+        check("msp_spgemm_radix_workspace",
+              lib().msp_spgemm_radix_workspace(ctypes.byref(self.a), ctypes.byref(self.b), ctypes.byref(self.info),
+                                               ctypes.byref(n)))
+        self.wsr = workspace(int(n.value), self.A.device, "spgemm_radix", self.stream)
+        nnz = ctypes.c_int64(0)
+        check("msp_spgemm_radix_symbolic",
+              lib().msp_spgemm_radix_symbolic(ctypes.byref(self.a), ctypes.byref(self.b), self.ws1.data_ptr(),
+                                              self.ws1.numel(), self.wsr.data_ptr(), self.wsr.numel(),
+                                              ctypes.byref(self.info), self.rp.data_ptr(), ctypes.byref(nnz),
+                                              _stream_ptr(self.A.device, self.stream)))
+        _claim(self.token, self.A.device, ("spgemm_setup", "spgemm_radix"), self.stream)
+        self.nnz = int(nnz.value)
+        return self.nnz
+
+    def numeric(self, col: torch.Tensor | None = None, val: torch.Tensor | None = None) -> CsrTensor:
+        if self.nnz is None or not _owns(self.token, self.A.device, ("spgemm_setup", "spgemm_radix"), self.stream):
+            self.symbolic()
+        dev = self.A.device
+        col = col if col is not None else torch.empty(self.nnz, dtype=torch.int32, device=dev)
+        val = val if val is not None else torch.empty(self.nnz, dtype=self.A.dtype, device=dev)
+        check("msp_spgemm_radix_numeric",
+              lib().msp_spgemm_radix_numeric(ctypes.byref(self.a), ctypes.byref(self.b), self.ws1.data_ptr(),
+                                             self.ws1.numel(), self.wsr.data_ptr(), self.wsr.numel(),
+                                             ctypes.byref(self.info), self.rp.data_ptr(),
+                                             col.data_ptr() if self.nnz else None,
+                                             val.data_ptr() if self.nnz else None, _stream_ptr(dev, self.stream)))
+        return CsrTensor(self.rp, col, val, (self.A.shape[0], self.B.shape[1]))
+
+
 def spgemm(A: CsrTensor, B: CsrTensor, stream=None) -> CsrTensor:
     """C = A B (expand / sort / compress)."""
     p = SpGemmPlan(A, B, stream)
