@@ -64,7 +64,7 @@
 extern "C" {
 #endif
 
-#define MSP_VERSION 2  /* 2: msp_spgemm_info passed to symbolic / numeric */
+#define MSP_VERSION 3  /* 2: msp_spgemm_info passed to symbolic / numeric; 3: segmented_rows */
 
 typedef enum {
     MSP_OK = 0,
@@ -194,6 +194,11 @@ typedef struct {
     int64_t long_chunks;     /* sorted chunks of the long-row pass */
     int64_t max_tile_span;   /* largest row span of a product tile: -1 after
                                 setup, set by symbolic (picks the key width) */
+    int64_t segmented_rows;  /* long rows taking the segmented (row-wise dense
+                                accumulator) path instead of the ESC long-row
+                                pass: output span <= 12288 columns and >= 1
+                                product per 4 columns of it (
+                                MSP_SPGEMM_SEGMENTED=0 disables) */
 } msp_spgemm_info;
 
 msp_status msp_spgemm_setup_workspace(const msp_csr *A, const msp_csr *B, size_t *bytes);

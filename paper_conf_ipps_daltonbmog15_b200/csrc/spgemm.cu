@@ -28,6 +28,7 @@
 //     (merge path per thread, stable) until one run per row remains; a head-
 //     flag pass reduces equal columns (counts, or scan + sums for numeric).
 #include <algorithm>
+#include <cstdlib>
 #include <climits>
 #include <cstdint>
 #include <cstdio>
@@ -110,6 +111,149 @@ __global__ void long_scatter_kernel(int32_t m, const int32_t *__restrict__ rp, c
     }
 }
 
+// ---------------------------------------------------- segmented path (f3)
+// The paper's future work: "adaptively introducing segmented
+// approaches when necessary" for rows where sorting the expanded products
+// gains little -- its failure case is Dense, whose rows produce few
+// duplicates per CTA but need huge temporary storage in the global pass
+// (P:1648-1660).  A long row whose output columns span at most SPA_W
+// columns, with at least one product per 4 columns of that span, is instead
+// accumulated row-wise in a shared-memory dense accumulator (one CTA per
+// row): no expanded product is stored, and the sum runs over k in A's
+// column order -- the order of Gustavson's oracle -- with separate multiply
+// and add roundings.
+constexpr int SPA_W = 12288;    // accumulator columns (96 KB fp64 + a bit per column)
+constexpr int SPA_NT = 256;
+
+__global__ void span_init_kernel(int32_t m, int32_t *__restrict__ lo, int32_t *__restrict__ hi)
+{
+    for (int64_t r = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; r < m; r += int64_t(gridDim.x) * blockDim.x) {
+        lo[r] = INT_MAX;
+        hi[r] = -1;
+    }
+}
+
+// column span of every long row: min / max over its products' columns
+__global__ void span_kernel(int64_t nnzA, const int32_t *__restrict__ Acol, const int32_t *__restrict__ arow,
+                            const uint8_t *__restrict__ rowlong, const int32_t *__restrict__ Brp,
+                            const int32_t *__restrict__ Bcol, int32_t *__restrict__ lo, int32_t *__restrict__ hi)
+{
+    for (int64_t j = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; j < nnzA; j += int64_t(gridDim.x) * blockDim.x) {
+        const int32_t r = arow[j];
+        if (!rowlong[r]) continue;
+        const int32_t k = Acol[j], b0 = Brp[k], b1 = Brp[k + 1];
+        if (b1 > b0) {
+            atomicMin(&lo[r], Bcol[b0]);
+            atomicMax(&hi[r], Bcol[b1 - 1]);
+        }
+    }
+}
+
+// cost model: segmented iff span <= SPA_W and P_r >= span / 4
+__global__ void spa_classify_kernel(int32_t m, const int32_t *__restrict__ rp, const int64_t *__restrict__ S,
+                                    const int32_t *__restrict__ lo, const int32_t *__restrict__ hi,
+                                    uint8_t *__restrict__ rowlong, int32_t *__restrict__ longflag,
+                                    int32_t *__restrict__ spaflag)
+{
+    for (int64_t r = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; r < m; r += int64_t(gridDim.x) * blockDim.x) {
+        int f = 0;
+        if (rowlong[r]) {
+            const int64_t span = int64_t(hi[r]) - lo[r] + 1;
+            const int64_t P = S[rp[r + 1]] - S[rp[r]];
+            if (span >= 1 && span <= SPA_W && 4 * P >= span) {
+                f = 1;
+                rowlong[r] = 2;   // masked in tiles like a long row
+                longflag[r] = 0;  // not in the ESC long-row pass
+            }
+        }
+        spaflag[r] = f;
+    }
+}
+
+__global__ void spa_scatter_kernel(int32_t m, const int32_t *__restrict__ spaflag, const int64_t *__restrict__ spapos,
+                                   int32_t *__restrict__ sparow)
+{
+    for (int64_t r = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; r < m; r += int64_t(gridDim.x) * blockDim.x)
+        if (spaflag[r]) sparow[spapos[r]] = int32_t(r);
+}
+
+// One CTA per segmented row.  Symbolic marks the row's output columns (no
+// ordering needed) and counts them; numeric accumulates a_ik * b_kj for k in
+// A's column order (a barrier per A nonzero keeps every column's sum in that
+// order), then writes the marked columns ascending at C.rp[r].
+template <typename V, bool NUM>
+__global__ void __launch_bounds__(SPA_NT)
+spa_row_kernel(const int32_t *__restrict__ sparow, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
+               const V *__restrict__ Aval, const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
+               const V *__restrict__ Bval, const int32_t *__restrict__ spanlo, const int32_t *__restrict__ spanhi,
+               int32_t *__restrict__ Crp_counts, const int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol,
+               V *__restrict__ Cval)
+{
+    extern __shared__ __align__(16) char spa_smem[];
+    double *acc = reinterpret_cast<double *>(spa_smem);                       // [SPA_W] (numeric)
+    uint32_t *mark = reinterpret_cast<uint32_t *>(spa_smem + (NUM ? SPA_W * 8 : 0));  // [SPA_W / 32]
+    __shared__ int32_t wsum[SPA_NT / 32];
+    const int tid = threadIdx.x;
+    const int32_t r = sparow[blockIdx.x];
+    const int32_t c0 = spanlo[r];
+    const int span = spanhi[r] - c0 + 1;
+    const int nw = (span + 31) >> 5;
+    for (int i = tid; i < nw; i += SPA_NT) mark[i] = 0u;
+    __syncthreads();
+    const int32_t a0 = Arp[r], a1 = Arp[r + 1];
+    for (int32_t j = a0; j < a1; ++j) {
+        const int32_t k = Acol[j];
+        const int32_t b0 = Brp[k], b1 = Brp[k + 1];
+        double a = 0.0;
+        if constexpr (NUM) a = double(Aval[j]);
+        for (int32_t q = b0 + tid; q < b1; q += SPA_NT) {
+            const int c = Bcol[q] - c0;
+            if constexpr (NUM) {
+                const double p = __dmul_rn(a, double(Bval[q]));
+                const uint32_t bit = 1u << (c & 31);
+                const bool seen = (mark[c >> 5] & bit) != 0;
+                acc[c] = seen ? __dadd_rn(acc[c], p) : p;
+                if (!seen) atomicOr(&mark[c >> 5], bit);
+            } else {
+                atomicOr(&mark[c >> 5], 1u << (c & 31));
+            }
+        }
+        if constexpr (NUM) __syncthreads();  // column sums advance in k order
+    }
+    __syncthreads();
+    // marked columns, ascending: thread t owns words [t*WPT, (t+1)*WPT)
+    constexpr int WPT = (SPA_W / 32 + SPA_NT - 1) / SPA_NT;
+    int cnt = 0;
+#pragma unroll
+    for (int u = 0; u < WPT; ++u) {
+        const int w = tid * WPT + u;
+        if (w < nw) cnt += __popc(mark[w]);
+    }
+    int tot;
+    int o = block_exclusive_sum<int, SPA_NT / 32>(cnt, wsum, 1, &tot);
+    if constexpr (!NUM) {
+        if (tid == 0) Crp_counts[r] = tot;
+    } else {
+        const int64_t base = int64_t(Crp[r]) + o;
+        int64_t p = base;
+#pragma unroll
+        for (int u = 0; u < WPT; ++u) {
+            const int w = tid * WPT + u;
+            if (w < nw) {
+                uint32_t bits = mark[w];
+                while (bits) {
+                    const int b = __ffs(bits) - 1;
+                    bits &= bits - 1;
+                    const int c = w * 32 + b;
+                    Ccol[p] = c0 + c;
+                    Cval[p] = V(acc[c]);
+                    ++p;
+                }
+            }
+        }
+    }
+}
+
 struct SetupWs {
     int32_t *arow;
     int64_t *S;          // [nnzA + 1]
@@ -121,7 +265,11 @@ struct SetupWs {
     int64_t *longO;      // [m + 1] prefix of longP
     int64_t *longC;      // [m]  chunks of the i-th long row
     int64_t *longCO;     // [m + 1] prefix of longC
-    unsigned long long *stats;  // [8]: [0] max row products, [1..5] gathered setup sizes
+    unsigned long long *stats;  // [8]: [0] max row products, [1..6] gathered setup sizes
+    int32_t *spanlo, *spanhi;   // [m] output column span of each long row (segmented path, f3)
+    int32_t *spaflag;           // [m] 1 = the row takes the segmented path
+    int64_t *spapos;            // [m + 1]
+    int32_t *sparow;            // [m] rows of the segmented path
     void *scan;
     size_t scan_bytes;
     size_t bytes;
@@ -143,6 +291,11 @@ SetupWs carve_setup(const msp_csr *A, void *ws, size_t cap, bool *ok)
     w.longC = cv.take<int64_t>(size_t(m > 0 ? m : 1));
     w.longCO = cv.take<int64_t>(size_t(m + 1));
     w.stats = cv.take<unsigned long long>(8);
+    w.spanlo = cv.take<int32_t>(size_t(m > 0 ? m : 1));
+    w.spanhi = cv.take<int32_t>(size_t(m > 0 ? m : 1));
+    w.spaflag = cv.take<int32_t>(size_t(m > 0 ? m : 1));
+    w.spapos = cv.take<int64_t>(size_t(m + 1));
+    w.sparow = cv.take<int32_t>(size_t(m > 0 ? m : 1));
     w.scan_bytes = scan_ws_bytes(std::max<int64_t>(std::max<int64_t>(m, nnz), 1));
     w.scan = cv.take<char>(w.scan_bytes);
     w.bytes = cv.off;
@@ -425,6 +578,11 @@ gemm_tile_kernel(const int32_t *__restrict__ Acol, const V *__restrict__ Aval, c
     const int nz = int(s1.j - j0), np = int(s1.p - p0);
     if (np == 0) return;
     const int32_t rbase = arow[j0];
+    {   // a tile inside one long / segmented row has nothing to do (its
+        // products are handled by the long-row or segmented pass)
+        const int64_t jl = (S[s1.j] < s1.p) ? s1.j : s1.j - 1;  // nonzero of the tile's last product
+        if (rowlong[rbase] && arow[jl] == rbase) return;
+    }
     // ---- expansion: merge path over (nonzero ends, products) of the tile ----
     {
         const int items = nz + np;
@@ -786,7 +944,7 @@ MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, void *ws, size_t cap, b
 }
 
 struct HostInfo {  // read back by setup (one synchronisation), passed to symbolic / numeric in msp_spgemm_info
-    int64_t nprods, nlong, LP, LC, maxP;
+    int64_t nprods, nlong, LP, LC, maxP, nspa;
 };
 
 // The setup sizes gathered into one device array (so setup reads them back
@@ -794,7 +952,8 @@ struct HostInfo {  // read back by setup (one synchronisation), passed to symbol
 // longCO[nlong], max row products.
 __global__ void info_gather_kernel(const int64_t *__restrict__ S, int64_t nnzA, const int64_t *__restrict__ longpos,
                                    int64_t m, const int64_t *__restrict__ longO, const int64_t *__restrict__ longCO,
-                                   const unsigned long long *__restrict__ stats, int64_t *__restrict__ out)
+                                   const unsigned long long *__restrict__ stats, const int64_t *__restrict__ spapos,
+                                   int64_t *__restrict__ out)
 {
     if (threadIdx.x != 0) return;
     const int64_t nlong = longpos[m];
@@ -803,6 +962,7 @@ __global__ void info_gather_kernel(const int64_t *__restrict__ S, int64_t nnzA, 
     out[2] = nlong > 0 ? longO[nlong] : 0;
     out[3] = nlong > 0 ? longCO[nlong] : 0;
     out[4] = int64_t(stats[0]);
+    out[5] = spapos[m];
 }
 
 // A pinned host staging word array per host thread for the synchronising reads.
@@ -825,18 +985,19 @@ msp_status read_back(const int64_t *dev, int n, int64_t *host, cudaStream_t s, c
 
 msp_status read_info(const SetupWs &sw, int64_t m, int64_t nnzA, HostInfo *h, cudaStream_t s)
 {
-    info_gather_kernel<<<1, 32, 0, s>>>(sw.S, nnzA, sw.longpos, m, sw.longO, sw.longCO, sw.stats,
+    info_gather_kernel<<<1, 32, 0, s>>>(sw.S, nnzA, sw.longpos, m, sw.longO, sw.longCO, sw.stats, sw.spapos,
                                         reinterpret_cast<int64_t *>(sw.stats) + 1);
     msp_status st = last_launch("info_gather_kernel");
     if (st != MSP_OK) return st;
-    int64_t v[5];
-    st = read_back(reinterpret_cast<const int64_t *>(sw.stats) + 1, 5, v, s, "spgemm: setup sizes");
+    int64_t v[6];
+    st = read_back(reinterpret_cast<const int64_t *>(sw.stats) + 1, 6, v, s, "spgemm: setup sizes");
     if (st != MSP_OK) return st;
     h->nprods = v[0];
     h->nlong = v[1];
     h->LP = v[2];
     h->LC = v[3];
     h->maxP = v[4];
+    h->nspa = v[5];
     return MSP_OK;
 }
 
@@ -908,6 +1069,32 @@ msp_status run_long(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const
     return last_launch("long_emit_kernel");
 }
 
+bool spa_enabled()
+{
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("MSP_SPGEMM_SEGMENTED");  // 0 disables the f3 path (ablation)
+        v = (e && atoi(e) == 0) ? 0 : 1;
+    }
+    return v != 0;
+}
+
+template <typename V, bool NUM>
+msp_status run_spa(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const HostInfo &h, int32_t *Crp,
+                   int32_t *Ccol, void *Cval, cudaStream_t s)
+{
+    if (h.nspa <= 0) return MSP_OK;
+    auto kern = spa_row_kernel<V, NUM>;
+    const int smem = (NUM ? SPA_W * 8 : 0) + SPA_W / 8 + 64;
+    msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), smem, "spgemm: segmented smem");
+    if (st != MSP_OK) return st;
+    kern<<<unsigned(h.nspa), SPA_NT, smem, s>>>(sw.sparow, A->row_offsets, A->col_idx,
+                                                static_cast<const V *>(A->vals), B->row_offsets, B->col_idx,
+                                                static_cast<const V *>(B->vals), sw.spanlo, sw.spanhi,
+                                                NUM ? nullptr : Crp + 1, Crp, Ccol, static_cast<V *>(Cval));
+    return last_launch(NUM ? "spa_row_kernel<numeric>" : "spa_row_kernel<symbolic>");
+}
+
 int64_t ntiles_of(int64_t nnzA, int64_t nprods) { return ceil_div(nnzA + nprods > 0 ? nnzA + nprods : 1, GM_TP); }
 
 msp_status prepare_main(const msp_csr *A, const void *ws1, size_t b1, void *ws2, size_t b2, SetupWs *sw, MainWs *mw,
@@ -929,6 +1116,7 @@ HostInfo host_info(const msp_spgemm_info *info)
     h.LP = info->long_products;
     h.LC = info->long_chunks;
     h.maxP = info->max_row_products;
+    h.nspa = info->segmented_rows;
     return h;
 }
 
@@ -974,6 +1162,25 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
                                                w.stats);
         st = last_launch("rowclass_kernel");
         if (st != MSP_OK) return st;
+        // segmented path for long rows with a narrow output span (f3)
+        span_init_kernel<<<blocks, 256, 0, s>>>(A->nrows, w.spanlo, w.spanhi);
+        st = last_launch("span_init_kernel");
+        if (st != MSP_OK) return st;
+        if (nnz > 0 && spa_enabled()) {
+            span_kernel<<<unsigned(std::min<int64_t>(ceil_div(nnz, 256), 148 * 16)), 256, 0, s>>>(
+                nnz, A->col_idx, w.arow, w.rowlong, B->row_offsets, B->col_idx, w.spanlo, w.spanhi);
+            st = last_launch("span_kernel");
+            if (st != MSP_OK) return st;
+        }
+        spa_classify_kernel<<<blocks, 256, 0, s>>>(A->nrows, A->row_offsets, w.S, w.spanlo, w.spanhi, w.rowlong,
+                                                   w.longflag, w.spaflag);
+        st = last_launch("spa_classify_kernel");
+        if (st != MSP_OK) return st;
+        st = scan_i32_to_i64(w.spaflag, w.spapos, m, w.scan, w.scan_bytes, s);
+        if (st != MSP_OK) return st;
+        spa_scatter_kernel<<<blocks, 256, 0, s>>>(A->nrows, w.spaflag, w.spapos, w.sparow);
+        st = last_launch("spa_scatter_kernel");
+        if (st != MSP_OK) return st;
         st = scan_i32_to_i64(w.longflag, w.longpos, m, w.scan, w.scan_bytes, s);
         if (st != MSP_OK) return st;
         st = cuda_check(cudaMemsetAsync(w.longC, 0, size_t(m) * sizeof(int64_t), s), "spgemm: clear");
@@ -988,6 +1195,7 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
         if (st != MSP_OK) return st;
     } else {
         st = cuda_check(cudaMemsetAsync(w.longpos, 0, sizeof(int64_t), s), "spgemm: clear");
+        if (st == MSP_OK) st = cuda_check(cudaMemsetAsync(w.spapos, 0, sizeof(int64_t), s), "spgemm: clear");
         if (st != MSP_OK) return st;
     }
     HostInfo h;
@@ -1004,6 +1212,7 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
     info->main_ws_bytes = int64_t(mw.bytes + 256);
     info->long_chunks = h.LC;
     info->max_tile_span = -1;  // set by symbolic
+    info->segmented_rows = h.nspa;
     return MSP_OK;
 }
 
@@ -1057,6 +1266,9 @@ msp_status spgemm_pass(const msp_csr *A, const msp_csr *B, const void *ws1, size
         if (st != MSP_OK) return st;
         st = (A->dtype == MSP_F64) ? run_long<double, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s)
                                    : run_long<float, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s);
+        if (st != MSP_OK) return st;
+        st = (A->dtype == MSP_F64) ? run_spa<double, NUM>(A, B, sw, h, Crp, Ccol, Cval, s)
+                                   : run_spa<float, NUM>(A, B, sw, h, Crp, Ccol, Cval, s);
         if (st != MSP_OK) return st;
     }
     if (!NUM) {
