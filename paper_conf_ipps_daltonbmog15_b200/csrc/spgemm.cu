@@ -138,13 +138,35 @@ __global__ void span_kernel(int64_t nnzA, const int32_t *__restrict__ Acol, cons
                             const uint8_t *__restrict__ rowlong, const int32_t *__restrict__ Brp,
                             const int32_t *__restrict__ Bcol, int32_t *__restrict__ lo, int32_t *__restrict__ hi)
 {
-    for (int64_t j = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; j < nnzA; j += int64_t(gridDim.x) * blockDim.x) {
-        const int32_t r = arow[j];
-        if (!rowlong[r]) continue;
-        const int32_t k = Acol[j], b0 = Brp[k], b1 = Brp[k + 1];
-        if (b1 > b0) {
-            atomicMin(&lo[r], Bcol[b0]);
-            atomicMax(&hi[r], Bcol[b1 - 1]);
+    // grid-stride with whole warps, so that a warp whose 32 nonzeros all
+    // belong to one long row (C4's dense row: 10^6 of them) reduces them
+    // first and issues ONE atomic pair instead of 32
+    const int64_t stride = int64_t(gridDim.x) * blockDim.x;
+    for (int64_t j0 = int64_t(blockIdx.x) * blockDim.x; j0 < nnzA; j0 += stride) {
+        const int64_t j = j0 + threadIdx.x;
+        int32_t r = -1, cl = INT_MAX, ch = -1;
+        if (j < nnzA) {
+            r = arow[j];
+            if (rowlong[r]) {
+                const int32_t k = Acol[j], b0 = Brp[k], b1 = Brp[k + 1];
+                if (b1 > b0) {
+                    cl = Bcol[b0];
+                    ch = Bcol[b1 - 1];
+                }
+            } else {
+                r = -1;
+            }
+        }
+        const int32_t r0 = __shfl_sync(0xffffffffu, r, 0);
+        if (__all_sync(0xffffffffu, r == r0)) {
+            const int32_t wl = __reduce_min_sync(0xffffffffu, cl), wh = __reduce_max_sync(0xffffffffu, ch);
+            if ((threadIdx.x & 31) == 0 && r0 >= 0 && wh >= 0) {
+                atomicMin(&lo[r0], wl);
+                atomicMax(&hi[r0], wh);
+            }
+        } else if (r >= 0 && ch >= 0) {
+            atomicMin(&lo[r], cl);
+            atomicMax(&hi[r], ch);
         }
     }
 }

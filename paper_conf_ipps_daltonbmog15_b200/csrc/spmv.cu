@@ -698,6 +698,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             const int slot = t & (RING - 1);
             const int rs = t % C::RSLOTS;
             const int tile_is = nx_is, z = nx_z;
+            if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 8 : 4);  // tile's gathers issued earlier
             // ---- phase A finish: products -> warp-private buffer ----
 #pragma unroll
             for (int u = 0; u < K; ++u) wprod[swz<K>(lane + 32 * u)] = double(vv[u]) * double(xv[u]);
@@ -707,9 +708,11 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             // run-ahead raised memory contention and per-CTA tail variance)
             // workers in lockstep: a warp that runs ahead would take issue slots from
             // the slowest one, whose lag then eats the ring's slack (measured)
+            if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 9 : 5);  // products formed
             named_bar_sync(1, NW * 32);
             if (lane == 0) mbar_arrive(&empty[stage]);
             mbar_wait(&rowsrdy[rs], (t / C::RSLOTS) & 1);
+            if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 13 : 12);  // lockstep + row map
             // ---- walk ----
             const uint32_t *flags = reinterpret_cast<const uint32_t *>(rslots + size_t(rs) * C::RSLOT_BYTES);
             const uint16_t *rmap =
@@ -800,7 +803,9 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                 }
             }
             // next tile's gathers fly while the previous tile's first row is finished
+            if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 10 : 6);  // walked + scanned
             if (t + 1 < ntiles) a_issue(t + 1);
+            if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 11 : 7);  // next tile's gathers issued
             // ---- the warp's first row of tile t-1 (deferred one tile so that
             //      the look-back never waits): carry of earlier warps (nearest
             //      first), then of earlier tiles ----
