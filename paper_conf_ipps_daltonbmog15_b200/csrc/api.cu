@@ -57,6 +57,19 @@ int sm_count()
     return cache[dev];
 }
 
+int64_t l2_bytes()
+{
+    static int64_t cache[64] = {0};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return int64_t(126) << 20;
+    if (!cache[dev]) {
+        int n = 0;
+        if (cudaDeviceGetAttribute(&n, cudaDevAttrL2CacheSize, dev) != cudaSuccess || n <= 0) n = 126 << 20;
+        cache[dev] = n;
+    }
+    return cache[dev];
+}
+
 // Pinned host words per host thread for the synchronising size read-backs
 // (a pageable destination would stage each small copy through a driver
 // buffer).  Never freed: one small allocation per host thread.

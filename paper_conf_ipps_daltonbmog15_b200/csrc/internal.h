@@ -15,6 +15,7 @@ void clear_error();
 
 // device properties of the current device (cached)
 int sm_count();
+int64_t l2_bytes();  // L2 cache size of the current device
 
 // returns MSP_OK or MSP_ERR_CUDA with the error text recorded
 msp_status cuda_check(cudaError_t e, const char *where);

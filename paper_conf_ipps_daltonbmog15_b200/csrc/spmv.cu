@@ -179,6 +179,41 @@ __device__ __forceinline__ double ldg_x(const float *p)
     return double(v);
 }
 
+// x gather of the transpose walk: ld.global.cg.L2::64B -- L2 only (no L1
+// line allocation: the walk serves irregular matrices, whose gathers rarely
+// reuse an L1 line; 3-7 % faster than __ldg on C3/C4/C5), and a 64-byte
+// L2 fill instead of the 128-byte line an L1 miss requests by default: a
+// random 8-byte gather from a DRAM-resident x then costs 65 instead of
+// 121 DRAM bytes (tools/probe/gather_probe.py; C5 13.0 -> 12.7 ms).
+// (profiles/r2/spmv_irregular_shapes.txt)  Experiment builds:
+// -DMSP_SPMV_GATHER=0 -> __ldg, 1 -> ld.global.cg, 2 -> ld.global.cs.
+#ifndef MSP_SPMV_GATHER
+#define MSP_SPMV_GATHER 3
+#endif
+template <typename T>
+__device__ __forceinline__ T gather_x(const T *p)
+{
+#if MSP_SPMV_GATHER == 1
+    return __ldcg(p);
+#elif MSP_SPMV_GATHER == 2
+    return __ldcs(p);
+#elif MSP_SPMV_GATHER == 3
+    T v;
+    if constexpr (sizeof(T) == 8) {
+        double d;
+        asm volatile("ld.global.cg.L2::64B.f64 %0, [%1];" : "=d"(d) : "l"(p));
+        v = T(d);
+    } else {
+        float f;
+        asm volatile("ld.global.cg.L2::64B.f32 %0, [%1];" : "=f"(f) : "l"(p));
+        v = T(f);
+    }
+    return v;
+#else
+    return __ldg(p);
+#endif
+}
+
 // Predicated global store (keeps the walk straight-line code).
 __device__ __forceinline__ void st_global_if(double *p, double v, bool pred)
 {
@@ -662,7 +697,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                 cidx[u] = int(c < col_lim ? c : 0u);
             }
 #pragma unroll
-            for (int u = 0; u < K; ++u) xv[u] = __ldg(x + cidx[u]);
+            for (int u = 0; u < K; ++u) xv[u] = gather_x(x + cidx[u]);
 #pragma unroll
             for (int u = 0; u < K; ++u) vv[u] = vs[lane + 32 * u];
         };
@@ -836,15 +871,32 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
     __syncthreads();
     if (!s_last) return;
     __threadfence();
+    // A row spanning many CTAs (C4's 10^6-nonzero row crosses ~100 CTA ranges
+    // at 8 CTAs/SM) is one run of equal carry keys: its head sums the run.
+    // The carries are staged in shared memory (the tile buffers, free now;
+    // the mbarrier words after them are not touched) so that the run sum
+    // is a shared-memory loop, not a chain of dependent L2 round trips.
+    constexpr int kStageBytes = C::SMEM - C::MISC_BYTES;
+    const bool staged = size_t(G) * (sizeof(int) + sizeof(double)) <= size_t(kStageBytes);
+    double *s_cv = reinterpret_cast<double *>(smem);
+    int *s_ck = reinterpret_cast<int *>(s_cv + G);
+    if (staged) {
+        for (int k = tid; k < G; k += blockDim.x) {
+            s_ck[k] = __ldcg(&recs[k].carry_key);
+            s_cv[k] = __ldcg(&recs[k].carry_val);
+        }
+        __syncthreads();
+    }
     for (int k = tid; k < G; k += blockDim.x) {
-        const int key = __ldcg(&recs[k].carry_key);
+        const int key = staged ? s_ck[k] : __ldcg(&recs[k].carry_key);
         if (key < 0 || key >= m) continue;
-        if (k > 0 && __ldcg(&recs[k - 1].carry_key) == key) continue;  // not the head of a run
+        if (k > 0 && (staged ? s_ck[k - 1] : __ldcg(&recs[k - 1].carry_key)) == key) continue;  // not a run head
         double s = 0.0;
         int k2 = k;
-        while (k2 < G && __ldcg(&recs[k2].carry_key) == key) {
-            s += __ldcg(&recs[k2].carry_val);
-            ++k2;
+        if (staged) {
+            for (; k2 < G && s_ck[k2] == key; ++k2) s += s_cv[k2];
+        } else {
+            for (; k2 < G && __ldcg(&recs[k2].carry_key) == key; ++k2) s += __ldcg(&recs[k2].carry_val);
         }
         // the CTA after the run emits row `key` first (continuity of the path)
         if (k2 < G && __ldcg(&recs[k2].head_row) == key) y[key] = V(s + __ldcg(&recs[k2].head_val));
@@ -853,14 +905,16 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
 }
 
 // Tile shapes (consumer threads, products per thread, stages, CTAs/SM).
-// Config 0 is the default; MSP_SPMV_CFG=<n> selects another (tuning only).
+// Configs 0 and 4 are the defaults (see launch()); MSP_SPMV_CFG=<n> forces one (tuning only).
 template <typename V, int I> struct Shape;
 template <typename V> struct Shape<V, 0> { using C = Cfg<V, 8, 2, 2, 2>; };
 template <typename V> struct Shape<V, 1> { using C = Cfg<V, 8, 2, 2, 3>; };
 template <typename V> struct Shape<V, 2> { using C = Cfg<V, 8, 3, 3, 2>; };
 template <typename V> struct Shape<V, 3> { using C = Cfg<V, 8, 2, 4, 2>; };
 template <typename V> struct Shape<V, 4> { using C = Cfg<V, 4, 2, 4, 4>; };
-constexpr int kNumShapes = 5;
+template <typename V> struct Shape<V, 5> { using C = Cfg<V, 4, 2, 4, 5>; };
+template <typename V> struct Shape<V, 6> { using C = Cfg<V, 2, 2, 4, 8>; };
+constexpr int kNumShapes = 7;
 
 template <typename V, class C>
 msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
@@ -869,7 +923,7 @@ msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t
     int occ = 1;
     msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), C::SMEM, "spmv: smem", C::THREADS, &occ);
     if (st != MSP_OK) return st;
-    if (occ > 4) occ = 4;
+    if (occ > 8) occ = 8;
     static bool said = false;
     if (!said && getenv("MSP_VERBOSE")) {
         fprintf(stderr, "msp spmv: rowk=%d K=%d NW=%d T=%d stages=%d smem=%d occupancy=%d CTAs/SM\n", int(C::ROWK),
@@ -962,8 +1016,17 @@ template <typename V>
 msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
 {
     int shape = shape_choice();
-    if (shape == -3)  // default: row-aligned lanes for long regular rows, transpose walk otherwise
-        shape = (A->nrows > 0 && double(A->nnz) >= 20.0 * double(A->nrows)) ? -1 : 0;
+    if (shape == -3) {
+        // default: row-aligned lanes for long regular rows; else the transpose
+        // walk, with 4 small CTAs per SM (T = 1,024) while x fits in half of
+        // L2 -- the x gathers are then L2-latency-bound and more resident
+        // tiles hide it (C3 686 -> 534 us, C4 106 -> 103 us) -- and 2 large
+        // CTAs per SM once x spills to DRAM, where more gathers in flight only
+        // add DRAM contention (C5 13.0 vs 13.3 ms).
+        // (profiles/r2/spmv_irregular_shapes.txt)
+        if (A->nrows > 0 && double(A->nnz) >= 20.0 * double(A->nrows)) shape = -1;
+        else shape = int64_t(A->ncols) * int64_t(sizeof(V)) <= l2_bytes() / 2 ? 4 : 0;
+    }
     switch (shape) {
     case -1: {
         const int K = k_choice(A);
@@ -975,6 +1038,8 @@ msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_
     case 2: return launch_cfg<V, typename Shape<V, 2>::C>(A, x, y, ws, ws_bytes, s);
     case 3: return launch_cfg<V, typename Shape<V, 3>::C>(A, x, y, ws, ws_bytes, s);
     case 4: return launch_cfg<V, typename Shape<V, 4>::C>(A, x, y, ws, ws_bytes, s);
+    case 5: return launch_cfg<V, typename Shape<V, 5>::C>(A, x, y, ws, ws_bytes, s);
+    case 6: return launch_cfg<V, typename Shape<V, 6>::C>(A, x, y, ws, ws_bytes, s);
     default: return launch_cfg<V, typename Shape<V, 0>::C>(A, x, y, ws, ws_bytes, s);
     }
 }
@@ -983,9 +1048,9 @@ msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_
 
 size_t spmv_ws_bytes(const msp_csr *A)
 {
-    // counter + one record per CTA (grid <= max(4 per SM, tiles / tiles-per-CTA))
+    // counter + one record per CTA (grid <= max(8 per SM, tiles / tiles-per-CTA))
     const int64_t tiles = ceil_div(int64_t(A->nrows) + A->nnz, 1024);
-    const int64_t g = std::max<int64_t>(int64_t(4) * sm_count(), ceil_div(tiles, 2));
+    const int64_t g = std::max<int64_t>(int64_t(8) * sm_count(), ceil_div(tiles, 2));
     return 512 + size_t(g) * sizeof(CtaRecord);
 }
 

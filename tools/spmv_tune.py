@@ -22,6 +22,8 @@ if os.path.exists(cache):
 else:
     A = gen.config(cfg, 'random')
     np.savez(cache, m=A.m, n=A.n, rp=A.rp, col=A.col, val=A.val)
+if os.environ.get('TUNE_DTYPE'):  # same structure, other value type (tuning aid)
+    A = gen.CSR(A.m, A.n, A.rp, A.col, A.val.astype(os.environ['TUNE_DTYPE']))
 x = gen.x_vector(A.n, 'random', seed=1000 + int(cfg[1]), dtype=A.val.dtype)
 dA = msp.CsrTensor.from_arrays(A.rp, A.col, A.val, (A.m, A.n), 'cuda')
 dx = torch.as_tensor(x, device='cuda')
