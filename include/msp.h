@@ -64,7 +64,7 @@
 extern "C" {
 #endif
 
-#define MSP_VERSION 3  /* 2: msp_spgemm_info passed to symbolic / numeric; 3: segmented_rows */
+#define MSP_VERSION 4  /* 2: msp_spgemm_info passed to symbolic / numeric; 3: segmented_rows; 4: msp_set_operation_async, msp_spadd_fused */
 
 typedef enum {
     MSP_OK = 0,
@@ -155,6 +155,23 @@ msp_status msp_spadd_symbolic(const msp_csr *A, const msp_csr *B, int32_t *C_row
 msp_status msp_spadd_numeric(const msp_csr *A, const msp_csr *B, const int32_t *C_row_offsets,
                              int32_t *C_col_idx, void *C_vals, void *ws, size_t ws_bytes,
                              void *stream);
+
+/* One-pass SpAdd (B200 design; same result as symbolic +
+ * numeric, bit for bit): the two phases of P:816-838 fused into one tile
+ * pass.  Each tile's output offset comes from a decoupled look-back over
+ * the tiles' output counts (the tiles' runs of C are contiguous in merge
+ * order), and C_row_offsets[r+1] is written at row r's row-end
+ * item.  The price is the allocation: C_col_idx / C_vals must hold
+ * C_capacity >= nnz(A) + nnz(B) entries (the union's upper bound; else
+ * MSP_ERR_SHAPE); C_row_offsets is device int32 [nrows+1].  *nnzC_host
+ * receives nnz(C); entries past it are unspecified.  Synchronises the
+ * stream.  MSP_ERR_OVERFLOW if nnz(C) > INT32_MAX; MSP_ERR_INPUT if the
+ * row-end total and the tile total disagree (unsorted or duplicate
+ * columns; stores stay inside C_capacity).  ws: msp_spadd_workspace()
+ * bytes. */
+msp_status msp_spadd_fused(const msp_csr *A, const msp_csr *B, int32_t *C_row_offsets,
+                           int32_t *C_col_idx, void *C_vals, int64_t C_capacity, int64_t *nnzC_host,
+                           void *ws, size_t ws_bytes, void *stream);
 
 /* ------------------------------------------------------------------------
  * SpGEMM  C = A B    (ESC: expansion, sorting, compression, P:256-262,
@@ -285,6 +302,21 @@ msp_status msp_set_operation(msp_set_op op, const void *A_keys, const void *A_va
                              const void *B_keys, const void *B_vals, int64_t nB, int32_t key_bytes,
                              int32_t val_bytes, void *C_keys, void *C_vals, int64_t C_capacity,
                              int64_t *nC_host, void *ws, size_t ws_bytes, void *stream);
+
+/* The same operation without the host round trip: nC_dev is a DEVICE
+ * int64[2] (8-byte aligned, caller-owned) that receives, in stream order,
+ * nC_dev[0] = the result size and nC_dev[1] != 0 iff the keys were found
+ * unsorted (the MSP_ERR_INPUT condition of msp_set_operation, which this
+ * call cannot return).  Async: two launches (partition, which also clears
+ * the look-back state, and the tile kernel), no stream synchronisation, no
+ * device-to-host copy -- for pipelines that consume the result on the GPU
+ * (e.g. a size-bounded next step reading nC_dev) and for the Fig 2 rate
+ * without the per-call host sync.  ws must stay reserved until the stream
+ * reaches the end of the call. */
+msp_status msp_set_operation_async(msp_set_op op, const void *A_keys, const void *A_vals, int64_t nA,
+                                   const void *B_keys, const void *B_vals, int64_t nB, int32_t key_bytes,
+                                   int32_t val_bytes, void *C_keys, void *C_vals, int64_t C_capacity,
+                                   int64_t *nC_dev, void *ws, size_t ws_bytes, void *stream);
 
 /* ------------------------------------------------------------------------
  * Multi-GPU helpers.  Row blocks are balanced by nnz:

@@ -23,11 +23,11 @@ STATUS = {0: "MSP_OK", 1: "MSP_ERR_ARG", 2: "MSP_ERR_DTYPE", 3: "MSP_ERR_SHAPE",
 EXPORTS = [
     "msp_status_string", "msp_last_error", "msp_version", "msp_launch_count",
     "msp_spmv_workspace", "msp_spmv", "msp_spmv_nnz_split_workspace", "msp_spmv_nnz_split",
-    "msp_spadd_workspace", "msp_spadd_symbolic", "msp_spadd_numeric",
+    "msp_spadd_workspace", "msp_spadd_symbolic", "msp_spadd_numeric", "msp_spadd_fused",
     "msp_spgemm_setup_workspace", "msp_spgemm_setup", "msp_spgemm_symbolic", "msp_spgemm_numeric",
     "msp_spgemm_radix_workspace", "msp_spgemm_radix_symbolic", "msp_spgemm_radix_numeric",
     "msp_csr_check", "msp_row_split", "msp_rebase_offsets", "msp_gather_values",
-    "msp_set_op_workspace", "msp_set_operation",
+    "msp_set_op_workspace", "msp_set_operation", "msp_set_operation_async",
 ]
 
 
@@ -69,6 +69,7 @@ _SIGS = {
     "msp_spadd_workspace": (ctypes.c_int, [_csr_p, _csr_p, _P(_sz)]),
     "msp_spadd_symbolic": (ctypes.c_int, [_csr_p, _csr_p, _vp, _P(_i64), _vp, _sz, _vp]),
     "msp_spadd_numeric": (ctypes.c_int, [_csr_p, _csr_p, _vp, _vp, _vp, _vp, _sz, _vp]),
+    "msp_spadd_fused": (ctypes.c_int, [_csr_p, _csr_p, _vp, _vp, _vp, _i64, _P(_i64), _vp, _sz, _vp]),
     "msp_spgemm_setup_workspace": (ctypes.c_int, [_csr_p, _csr_p, _P(_sz)]),
     "msp_spgemm_setup": (ctypes.c_int, [_csr_p, _csr_p, _vp, _sz, _P(msp_spgemm_info), _vp]),
     "msp_spgemm_symbolic": (ctypes.c_int, [_csr_p, _csr_p, _vp, _sz, _vp, _sz, _P(msp_spgemm_info), _vp, _P(_i64),
@@ -87,6 +88,8 @@ _SIGS = {
     "msp_set_op_workspace": (ctypes.c_int, [_i64, _i64, _P(_sz)]),
     "msp_set_operation": (ctypes.c_int, [ctypes.c_int, _vp, _vp, _i64, _vp, _vp, _i64, _i32, _i32, _vp, _vp, _i64,
                                           _P(_i64), _vp, _sz, _vp]),
+    "msp_set_operation_async": (ctypes.c_int, [ctypes.c_int, _vp, _vp, _i64, _vp, _vp, _i64, _i32, _i32, _vp, _vp,
+                                                _i64, _vp, _vp, _sz, _vp]),
 }
 
 _lib = None

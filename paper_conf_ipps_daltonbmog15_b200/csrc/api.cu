@@ -315,6 +315,28 @@ msp_status msp_spadd_numeric(const msp_csr *A, const msp_csr *B, const int32_t *
     return spadd_numeric_run(A, B, C_row_offsets, C_col_idx, C_vals, ws, ws_bytes, as_stream(stream));
 }
 
+msp_status msp_spadd_fused(const msp_csr *A, const msp_csr *B, int32_t *C_row_offsets, int32_t *C_col_idx,
+                           void *C_vals, int64_t C_capacity, int64_t *nnzC_host, void *ws, size_t ws_bytes,
+                           void *stream)
+{
+    clear_error();
+    msp_status st = check_pair_add(A, B);
+    if (st != MSP_OK) return st;
+    if (!C_row_offsets || !nnzC_host || !ws) return MSP_ERR_ARG;
+    if (C_capacity < A->nnz + B->nnz) {
+        set_error("spadd fused: C capacity %lld below nnz(A) + nnz(B) = %lld", (long long)C_capacity,
+                  (long long)(A->nnz + B->nnz));
+        return MSP_ERR_SHAPE;
+    }
+    if (C_capacity > 0 && (!C_col_idx || !C_vals)) return MSP_ERR_ARG;
+    if (ws_bytes < spadd_ws_bytes(A, B)) return MSP_ERR_WORKSPACE;
+    st = debug_validate(A, 1, ws, ws_bytes, spadd_ws_bytes(A, B), as_stream(stream), "spadd A");
+    if (st == MSP_OK) st = debug_validate(B, 1, ws, ws_bytes, spadd_ws_bytes(A, B), as_stream(stream), "spadd B");
+    if (st != MSP_OK) return st;
+    return spadd_fused_run(A, B, C_row_offsets, C_col_idx, C_vals, C_capacity, nnzC_host, ws, ws_bytes,
+                           as_stream(stream));
+}
+
 // ------------------------------------------------------------------ SpGEMM
 static msp_status check_pair_mul(const msp_csr *A, const msp_csr *B)
 {
@@ -487,13 +509,12 @@ msp_status msp_set_op_workspace(int64_t nA, int64_t nB, size_t *bytes)
     return MSP_OK;
 }
 
-msp_status msp_set_operation(msp_set_op op, const void *A_keys, const void *A_vals, int64_t nA, const void *B_keys,
-                             const void *B_vals, int64_t nB, int32_t key_bytes, int32_t val_bytes, void *C_keys,
-                             void *C_vals, int64_t C_capacity, int64_t *nC_host, void *ws, size_t ws_bytes,
-                             void *stream)
+namespace {
+msp_status set_op_args(msp_set_op op, const void *A_keys, const void *A_vals, int64_t nA, const void *B_keys,
+                       const void *B_vals, int64_t nB, int32_t key_bytes, int32_t val_bytes, void *C_keys,
+                       void *C_vals, int64_t C_capacity, void *ws)
 {
-    clear_error();
-    if (!nC_host || nA < 0 || nB < 0 || int(op) < 0 || int(op) > 3) return MSP_ERR_ARG;
+    if (nA < 0 || nB < 0 || int(op) < 0 || int(op) > 3) return MSP_ERR_ARG;
     if (key_bytes != 4 && key_bytes != 8) {
         set_error("set op: key_bytes must be 4 or 8");
         return MSP_ERR_DTYPE;
@@ -520,9 +541,36 @@ msp_status msp_set_operation(msp_set_op op, const void *A_keys, const void *A_va
         return MSP_ERR_ARG;
     }
     if (!ws && nA + nB > 0) return MSP_ERR_ARG;
+    return MSP_OK;
+}
+}  // namespace
+
+msp_status msp_set_operation(msp_set_op op, const void *A_keys, const void *A_vals, int64_t nA, const void *B_keys,
+                             const void *B_vals, int64_t nB, int32_t key_bytes, int32_t val_bytes, void *C_keys,
+                             void *C_vals, int64_t C_capacity, int64_t *nC_host, void *ws, size_t ws_bytes,
+                             void *stream)
+{
+    clear_error();
+    if (!nC_host) return MSP_ERR_ARG;
+    msp_status st = set_op_args(op, A_keys, A_vals, nA, B_keys, B_vals, nB, key_bytes, val_bytes, C_keys, C_vals,
+                                C_capacity, ws);
+    if (st != MSP_OK) return st;
     return set_op_run(int(op), A_keys, A_vals, nA, B_keys, B_vals, nB, key_bytes, val_bytes, C_keys, C_vals, C_capacity,
-                      nC_host,
-                      ws, ws_bytes, as_stream(stream));
+                      nC_host, nullptr, ws, ws_bytes, as_stream(stream));
+}
+
+msp_status msp_set_operation_async(msp_set_op op, const void *A_keys, const void *A_vals, int64_t nA,
+                                   const void *B_keys, const void *B_vals, int64_t nB, int32_t key_bytes,
+                                   int32_t val_bytes, void *C_keys, void *C_vals, int64_t C_capacity, int64_t *nC_dev,
+                                   void *ws, size_t ws_bytes, void *stream)
+{
+    clear_error();
+    if (!nC_dev || (reinterpret_cast<uintptr_t>(nC_dev) & 7)) return MSP_ERR_ARG;
+    msp_status st = set_op_args(op, A_keys, A_vals, nA, B_keys, B_vals, nB, key_bytes, val_bytes, C_keys, C_vals,
+                                C_capacity, ws);
+    if (st != MSP_OK) return st;
+    return set_op_run(int(op), A_keys, A_vals, nA, B_keys, B_vals, nB, key_bytes, val_bytes, C_keys, C_vals, C_capacity,
+                      nullptr, nC_dev, ws, ws_bytes, as_stream(stream));
 }
 
 }  // extern "C"

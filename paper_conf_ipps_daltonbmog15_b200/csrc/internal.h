@@ -79,6 +79,8 @@ msp_status spadd_symbolic_run(const msp_csr *A, const msp_csr *B, int32_t *Crp, 
                               size_t ws_bytes, cudaStream_t s);
 msp_status spadd_numeric_run(const msp_csr *A, const msp_csr *B, const int32_t *Crp, int32_t *Ccol, void *Cval,
                              void *ws, size_t ws_bytes, cudaStream_t s);
+msp_status spadd_fused_run(const msp_csr *A, const msp_csr *B, int32_t *Crp, int32_t *Ccol, void *Cval, int64_t cap,
+                           int64_t *nnzC, void *ws, size_t ws_bytes, cudaStream_t s);
 
 size_t spgemm_setup_ws_bytes(const msp_csr *A, const msp_csr *B);
 msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_t b1, msp_spgemm_info *info,
@@ -103,8 +105,8 @@ msp_status csr_check_run(const msp_csr *A, int sorted_unique, int32_t *flags_hos
                          cudaStream_t s);
 size_t set_op_ws_bytes(int64_t na, int64_t nb);
 msp_status set_op_run(int op, const void *A, const void *Av, int64_t na, const void *B, const void *Bv, int64_t nb,
-                      int key_bytes, int val_bytes, void *C, void *Cv, int64_t cap, int64_t *nC_host, void *ws,
-                      size_t ws_bytes, cudaStream_t s);
+                      int key_bytes, int val_bytes, void *C, void *Cv, int64_t cap, int64_t *nC_host, int64_t *nC_dev,
+                      void *ws, size_t ws_bytes, cudaStream_t s);
 msp_status gather_run(const void *src, const int32_t *idx, int64_t n, int value_bytes, void *dst, cudaStream_t s);
 msp_status rebase_run(const int32_t *in, int32_t *out, int64_t n, int64_t base, cudaStream_t s);
 

@@ -142,11 +142,18 @@ __device__ __forceinline__ Cut balanced_fixup(LA A, IT na, LB B, IT nb, const IT
 // probes per round cost more DRAM sectors than the binary search's latency.)
 template <typename KT>
 __global__ void set_partition_kernel(const KT *__restrict__ A, int64_t na, const KT *__restrict__ B, int64_t nb,
-                                     int64_t ntiles, Cut *__restrict__ cuts)
+                                     int64_t ntiles, Cut *__restrict__ cuts, uint64_t *__restrict__ states,
+                                     unsigned *__restrict__ ticket, int64_t *__restrict__ nC)
 {
     const int64_t total = na + nb;
+    // also clears the tile kernel's look-back state, ticket and result words
+    // (one launch fewer than a separate memset; the tile kernel runs after
+    // this one on the same stream)
+    if (blockIdx.x == 0 && threadIdx.x < 4) ticket[threadIdx.x] = 0u;
+    if (blockIdx.x == 0 && threadIdx.x < 2) nC[threadIdx.x] = 0;
     for (int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; k <= ntiles;
          k += int64_t(gridDim.x) * blockDim.x) {
+        if (k < ntiles) states[k] = 0ull;
         const int64_t d = k * SET_T < total ? k * SET_T : total;
         cuts[k] = balanced_cut<KT, int64_t>([&](int64_t x) { return A[x]; }, na, [&](int64_t x) { return B[x]; }, nb, d);
     }
@@ -437,33 +444,36 @@ size_t set_op_ws_bytes(int64_t na, int64_t nb)
 }
 
 msp_status set_op_run(int op, const void *A, const void *Av, int64_t na, const void *B, const void *Bv, int64_t nb,
-                      int key_bytes, int val_bytes, void *C, void *Cv, int64_t cap, int64_t *nC_host, void *ws,
-                      size_t ws_bytes, cudaStream_t s)
+                      int key_bytes, int val_bytes, void *C, void *Cv, int64_t cap, int64_t *nC_host, int64_t *nC_dev,
+                      void *ws, size_t ws_bytes, cudaStream_t s)
 {
     bool ok;
     SetWs w = carve(na, nb, ws, ws_bytes, &ok);
     if (!ok) return MSP_ERR_WORKSPACE;
+    if (nC_dev) w.nC = nC_dev;  // asynchronous form: the result words go to the caller's device buffer
     if (w.ntiles == 0) {
+        if (nC_dev) return cuda_check(cudaMemsetAsync(nC_dev, 0, 2 * sizeof(int64_t), s), "set op: empty result");
         *nC_host = 0;
         return MSP_OK;
     }
-    msp_status st = cuda_check(cudaMemsetAsync(ws, 0, reinterpret_cast<char *>(w.cuts) - static_cast<char *>(ws), s),
-                               "set op: clear look-back state");
-    if (st != MSP_OK) return st;
+    msp_status st;
     {
         const unsigned blocks = unsigned(std::min<int64_t>(ceil_div(w.ntiles + 1, 256), 148 * 8));
         if (key_bytes == 4)
             set_partition_kernel<uint32_t><<<blocks, 256, 0, s>>>(static_cast<const uint32_t *>(A), na,
-                                                                  static_cast<const uint32_t *>(B), nb, w.ntiles, w.cuts);
+                                                                  static_cast<const uint32_t *>(B), nb, w.ntiles, w.cuts,
+                                                                  w.states, w.ticket, w.nC);
         else
             set_partition_kernel<uint64_t><<<blocks, 256, 0, s>>>(static_cast<const uint64_t *>(A), na,
-                                                                  static_cast<const uint64_t *>(B), nb, w.ntiles, w.cuts);
+                                                                  static_cast<const uint64_t *>(B), nb, w.ntiles, w.cuts,
+                                                                  w.states, w.ticket, w.nC);
         st = last_launch("set_partition_kernel");
         if (st != MSP_OK) return st;
     }
     st = (key_bytes == 4) ? launch_kv<uint32_t>(op, val_bytes, A, Av, na, B, Bv, nb, w, C, Cv, cap, s)
                           : launch_kv<uint64_t>(op, val_bytes, A, Av, na, B, Bv, nb, w, C, Cv, cap, s);
     if (st != MSP_OK) return st;
+    if (nC_dev) return MSP_OK;
     // the result size comes back through a pinned word (a pageable
     // destination would stage the 8-byte copy through a driver buffer)
     static thread_local int64_t *pinned = nullptr;

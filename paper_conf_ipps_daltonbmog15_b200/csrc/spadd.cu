@@ -73,11 +73,16 @@ __device__ __forceinline__ void row_merge_path(LA Acol, int a_lo, int a_hi, LB B
 
 __global__ void spadd_partition_kernel(int32_t m, int64_t nnzA, int64_t nnzB, const int32_t *__restrict__ Arp,
                                        const int32_t *__restrict__ Acol, const int32_t *__restrict__ Brp,
-                                       const int32_t *__restrict__ Bcol, int64_t ntiles, Split *__restrict__ splits)
+                                       const int32_t *__restrict__ Bcol, int64_t ntiles, Split *__restrict__ splits,
+                                       uint64_t *__restrict__ states, unsigned *__restrict__ ticket)
 {
     const int64_t E = nnzA + nnzB;
     const int64_t total = int64_t(m) + E;
+    // fused form: clear the look-back state and the tile ticket (the fused
+    // tile kernel runs after this launch on the same stream)
+    if (states && blockIdx.x == 0 && threadIdx.x == 0) *ticket = 0u;
     for (int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; k <= ntiles; k += int64_t(gridDim.x) * blockDim.x) {
+        if (states && k < ntiles) states[k] = 0ull;
         const int64_t d = min(k * ADD_T, total);
         // rows: smallest i with NOT(R_end[i] <= d - i - 1)
         int64_t lo = max(int64_t(0), d - E), hi = min(d, int64_t(m));
@@ -160,21 +165,40 @@ __device__ __forceinline__ T *issue_stage(const Staged &st, const T *base, int64
     return reinterpret_cast<T *>(dst + st.w.first);
 }
 
-template <typename V, bool FILL>
+// Tile kernel modes: COUNT (symbolic: per-row unique counts), FILL (numeric:
+// writes C at the offsets the symbolic phase produced) and FUSED (one pass:
+// the tile's output offset comes from a decoupled look-back over the tiles'
+// output counts, and C.row_offsets from the row-end items -- DESIGN §4.2).
+enum AddMode { ADD_COUNT = 0, ADD_FILL = 1, ADD_FUSED = 2 };
+constexpr uint64_t AS_AGG = 1ull << 62, AS_PRE = 2ull << 62, AS_VAL = (1ull << 62) - 1;
+
+template <typename V, int MODE>
 __global__ void __launch_bounds__(ADD_NT)
 spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
                   const V *__restrict__ Aval, const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
                   const V *__restrict__ Bval, int64_t nnzA, int64_t nnzB, const Split *__restrict__ splits,
                   int32_t *__restrict__ tile_count, const int64_t *__restrict__ tile_off,
-                  int32_t *__restrict__ Crp_counts, int32_t *__restrict__ Ccol, V *__restrict__ Cval)
+                  int32_t *__restrict__ Crp_counts, int32_t *__restrict__ Ccol, V *__restrict__ Cval,
+                  uint64_t *__restrict__ states, unsigned *__restrict__ ticket, int64_t *__restrict__ totals,
+                  int64_t ntiles, int64_t cap)
 {
+    constexpr bool FILL = MODE != ADD_COUNT;
+    constexpr bool FUSED = MODE == ADD_FUSED;
     using L = AddLayout<V, FILL>;
     extern __shared__ __align__(128) char smem_raw[];
     Split *S_st = reinterpret_cast<Split *>(smem_raw + L::ST_OFF);
     int32_t *S_wsum = reinterpret_cast<int32_t *>(smem_raw + L::WS_OFF);
     uint64_t *bar = reinterpret_cast<uint64_t *>(smem_raw + L::BAR_OFF);
+    __shared__ int s_tile;
+    __shared__ int64_t s_base;
     const int tid = threadIdx.x;
-    const int k = blockIdx.x;
+    int k = blockIdx.x;
+    if constexpr (FUSED) {
+        // tiles in claim order: the look-back never waits on an unstarted tile
+        if (tid == 0) s_tile = int(atomicAdd(ticket, 1u));
+        __syncthreads();
+        k = s_tile;
+    }
     const Split s0 = splits[k], s1 = splits[k + 1];
     const int r0 = s0.r, r1 = s1.r;
     const int ga0 = s0.a, gb0 = s0.b;
@@ -322,7 +346,7 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
         int cnt = 0;
         int rc[ADD_STEPS];
         V rv[ADD_STEPS];
-        unsigned em = 0;
+        unsigned em = 0, rem = 0;  // output steps, row-end steps
         if (regs) {
             int r = beg.r, ia = beg.a, ib = beg.b;
             int ah = (r < m) ? a_hi(r) : nA, bh = (r < m) ? b_hi(r) : nB;
@@ -331,6 +355,7 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
                 if (r != end.r || ia != end.a || ib != end.b) {
                     const bool ra = ia < ah, rb = ib < bh;
                     if (!ra && !rb) {  // row-end item
+                        rem |= 1u << st;
                         ++r;
                         if (r < m) {
                             ah = a_hi(r);
@@ -358,33 +383,96 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
         }
         int tot;
         int o = block_exclusive_sum<int, ADD_NT / 32>(cnt, S_wsum, 0, &tot);
+        const int o_thread = o;
+        if constexpr (FUSED) {
+            if (tid < 32) {  // decoupled look-back over the tiles' output counts (warp 0)
+                const int lane = tid;
+                int64_t excl = 0;
+                if (k == 0) {
+                    if (lane == 0)  // flag and value share one word: no fence needed
+                        atomicExch(reinterpret_cast<unsigned long long *>(&states[0]),
+                                   (unsigned long long)(AS_PRE | uint64_t(tot)));
+                } else {
+                    if (lane == 0)
+                        atomicExch(reinterpret_cast<unsigned long long *>(&states[k]),
+                                   (unsigned long long)(AS_AGG | uint64_t(tot)));
+                    for (int pos = k - 1;; pos -= 32) {
+                        const int q = pos - lane;
+                        uint64_t sw = AS_PRE;  // virtual prefix 0 before tile 0
+                        if (q >= 0) {
+                            do {
+                                sw = *reinterpret_cast<volatile uint64_t *>(&states[q]);
+                            } while ((sw & ~AS_VAL) == 0);  // predecessor not published yet
+                        }
+                        const unsigned pre = __ballot_sync(0xffffffffu, (sw & AS_PRE) != 0);
+                        const int stop = pre ? __ffs(pre) - 1 : 32;  // nearest predecessor with a prefix
+                        int64_t v = lane <= stop ? int64_t(sw & AS_VAL) : 0;
+#pragma unroll
+                        for (int d = 16; d > 0; d >>= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
+                        excl += v;
+                        if (pre) break;
+                    }
+                    if (lane == 0)
+                        atomicExch(reinterpret_cast<unsigned long long *>(&states[k]),
+                                   (unsigned long long)(AS_PRE | uint64_t(excl + tot)));
+                }
+                if (lane == 0) {
+                    s_base = excl;
+                    if (k == ntiles - 1) totals[1] = excl + tot;  // nnz(C) by the tiles
+                }
+            }
+        }
         if (regs) {
 #pragma unroll
             for (int st = 0; st < ADD_STEPS; ++st) {
-                if (em & (1u << st)) {
+                if ((em & (1u << st)) && o < ADD_T) {  // bound binds only on malformed input
                     ocol[o] = rc[st];
                     oval[o] = rv[st];
                     ++o;
                 }
             }
-        } else {  // fallback: the windows are still being read, store straight to C
-            int64_t p = tile_off[k] + o;
+        }
+        if constexpr (FUSED) __syncthreads();  // s_base published
+        int64_t tbase;
+        if constexpr (FUSED) tbase = s_base;
+        else tbase = tile_off[k];
+        if constexpr (FUSED) {
+            if (k == 0 && tid == 0) Crp_counts[0] = 0;
+            if (regs && rem) {  // C.row_offsets[r+1] at each row end of this thread's path
+                int r = beg.r, p = o_thread;
+#pragma unroll
+                for (int st = 0; st < ADD_STEPS; ++st) {
+                    if (rem & (1u << st)) {
+                        Crp_counts[r + 1] = int32_t(tbase + p);
+                        ++r;
+                    }
+                    p += (em >> st) & 1u;
+                }
+            }
+        }
+        if (!regs) {  // fallback: the windows are still being read, store straight to C
+            int64_t p = tbase + o_thread;
             walk(
                 [&](int c, int ia, int ib) {
                     V v;
                     if (ia >= 0 && ib >= 0) v = avs[ia] + bvs[ib];  // one rounding, A first (Alg. 1)
                     else v = (ia >= 0) ? avs[ia] : bvs[ib];
-                    Ccol[p] = c;
-                    Cval[p] = v;
+                    if (p < cap) {  // binds only on malformed (unsorted) input in the fused form
+                        Ccol[p] = c;
+                        Cval[p] = v;
+                    }
                     ++p;
                 },
-                [&](int) {});
+                [&](int r) {
+                    if constexpr (FUSED) Crp_counts[r + 1] = int32_t(p);
+                });
         }
         if (regs) {
             __syncthreads();
             // the tile's run of C is contiguous: coalesced stores
-            const int64_t base = tile_off[k];
-            for (int i = tid; i < tot; i += ADD_NT) {
+            const int64_t base = tbase;
+            const int nst = min(tot, ADD_T);  // binds only on malformed input
+            for (int i = tid; i < nst && base + i < cap; i += ADD_NT) {
                 Ccol[base + i] = ocol[i];
                 Cval[base + i] = oval[i];
             }
@@ -397,6 +485,8 @@ struct AddWs {
     int32_t *tile_count;
     int64_t *tile_off;  // [ntiles + 1]
     int64_t *totals;    // [4]
+    uint64_t *states;   // [ntiles] fused form: look-back status words
+    unsigned *ticket;   // [4]      fused form: tile claim counter
     void *scan;
     size_t scan_bytes;
     int64_t ntiles;
@@ -413,6 +503,8 @@ AddWs carve_ws(const msp_csr *A, const msp_csr *B, void *ws, size_t bytes, bool 
     w.tile_count = cv.take<int32_t>(size_t(w.ntiles));
     w.tile_off = cv.take<int64_t>(size_t(w.ntiles + 1));
     w.totals = cv.take<int64_t>(4);
+    w.states = cv.take<uint64_t>(size_t(w.ntiles));
+    w.ticket = cv.take<unsigned>(4);
     w.scan_bytes = scan_ws_bytes(std::max<int64_t>(A->nrows, w.ntiles));
     w.scan = cv.take<char>(w.scan_bytes);
     w.bytes = cv.off;
@@ -420,19 +512,32 @@ AddWs carve_ws(const msp_csr *A, const msp_csr *B, void *ws, size_t bytes, bool 
     return w;
 }
 
-template <typename V, bool FILL>
+template <typename V, int MODE>
 msp_status launch_tiles(const msp_csr *A, const msp_csr *B, const AddWs &w, int32_t *Crp, int32_t *Ccol, void *Cval,
-                        cudaStream_t s)
+                        int64_t cap, cudaStream_t s)
 {
-    auto kern = spadd_tile_kernel<V, FILL>;
-    const int smem = AddLayout<V, FILL>::BYTES;
+    auto kern = spadd_tile_kernel<V, MODE>;
+    const int smem = AddLayout<V, MODE != ADD_COUNT>::BYTES;
     msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), smem, "spadd: smem");
     if (st != MSP_OK) return st;
+    // COUNT adds row counts into Crp + 1; FUSED writes Crp[0 .. m] itself
+    int32_t *rp = Crp ? (MODE == ADD_FUSED ? Crp : Crp + 1) : nullptr;
     kern<<<unsigned(w.ntiles), ADD_NT, smem, s>>>(
         A->nrows, A->row_offsets, A->col_idx, static_cast<const V *>(A->vals), B->row_offsets, B->col_idx,
-        static_cast<const V *>(B->vals), A->nnz, B->nnz, w.splits, w.tile_count, w.tile_off, Crp ? Crp + 1 : nullptr, Ccol,
-        static_cast<V *>(Cval));
-    return last_launch(FILL ? "spadd_tile_kernel<fill>" : "spadd_tile_kernel<count>");
+        static_cast<const V *>(B->vals), A->nnz, B->nnz, w.splits, w.tile_count, w.tile_off, rp, Ccol,
+        static_cast<V *>(Cval), w.states, w.ticket, w.totals, w.ntiles, cap);
+    return last_launch(MODE == ADD_FUSED ? "spadd_tile_kernel<fused>"
+                                         : MODE == ADD_FILL ? "spadd_tile_kernel<fill>" : "spadd_tile_kernel<count>");
+}
+
+msp_status launch_partition(const msp_csr *A, const msp_csr *B, const AddWs &w, bool fused, cudaStream_t s)
+{
+    const int64_t n = w.ntiles + 1;
+    const unsigned blocks = unsigned(std::min<int64_t>(ceil_div(n, 256), 148 * 8));
+    spadd_partition_kernel<<<blocks, 256, 0, s>>>(A->nrows, A->nnz, B->nnz, A->row_offsets, A->col_idx,
+                                                  B->row_offsets, B->col_idx, w.ntiles, w.splits,
+                                                  fused ? w.states : nullptr, w.ticket);
+    return last_launch("spadd_partition_kernel");
 }
 
 }  // namespace
@@ -457,16 +562,10 @@ msp_status spadd_symbolic_run(const msp_csr *A, const msp_csr *B, int32_t *Crp, 
         *nnzC = 0;
         return cuda_check(cudaStreamSynchronize(s), "spadd: sync");
     }
-    {
-        const int64_t n = w.ntiles + 1;
-        const unsigned blocks = unsigned(std::min<int64_t>(ceil_div(n, 256), 148 * 8));
-        spadd_partition_kernel<<<blocks, 256, 0, s>>>(m, A->nnz, B->nnz, A->row_offsets, A->col_idx, B->row_offsets,
-                                                      B->col_idx, w.ntiles, w.splits);
-        st = last_launch("spadd_partition_kernel");
-        if (st != MSP_OK) return st;
-    }
-    st = (A->dtype == MSP_F64) ? launch_tiles<double, false>(A, B, w, Crp, nullptr, nullptr, s)
-                               : launch_tiles<float, false>(A, B, w, Crp, nullptr, nullptr, s);
+    st = launch_partition(A, B, w, false, s);
+    if (st != MSP_OK) return st;
+    st = (A->dtype == MSP_F64) ? launch_tiles<double, ADD_COUNT>(A, B, w, Crp, nullptr, nullptr, INT64_MAX, s)
+                               : launch_tiles<float, ADD_COUNT>(A, B, w, Crp, nullptr, nullptr, INT64_MAX, s);
     if (st != MSP_OK) return st;
     // row counts -> C.row_offsets (in place, Crp[0] stays 0); tile counts -> offsets
     st = scan_counts_to_offsets_i32(Crp + 1, m, &w.totals[0], w.scan, w.scan_bytes, s);
@@ -504,8 +603,52 @@ msp_status spadd_numeric_run(const msp_csr *A, const msp_csr *B, const int32_t *
     if (!ok) return MSP_ERR_WORKSPACE;
     (void)Crp;
     if (A->nrows == 0) return MSP_OK;
-    return (A->dtype == MSP_F64) ? launch_tiles<double, true>(A, B, w, nullptr, Ccol, Cval, s)
-                                 : launch_tiles<float, true>(A, B, w, nullptr, Ccol, Cval, s);
+    return (A->dtype == MSP_F64) ? launch_tiles<double, ADD_FILL>(A, B, w, nullptr, Ccol, Cval, INT64_MAX, s)
+                                 : launch_tiles<float, ADD_FILL>(A, B, w, nullptr, Ccol, Cval, INT64_MAX, s);
+}
+
+msp_status spadd_fused_run(const msp_csr *A, const msp_csr *B, int32_t *Crp, int32_t *Ccol, void *Cval, int64_t cap,
+                           int64_t *nnzC, void *ws, size_t ws_bytes, cudaStream_t s)
+{
+    bool ok;
+    AddWs w = carve_ws(A, B, ws, ws_bytes, &ok);
+    if (!ok) return MSP_ERR_WORKSPACE;
+    const int32_t m = A->nrows;
+    msp_status st;
+    if (m == 0) {
+        *nnzC = 0;
+        st = cuda_check(cudaMemsetAsync(Crp, 0, sizeof(int32_t), s), "spadd: rp");
+        if (st != MSP_OK) return st;
+        return cuda_check(cudaStreamSynchronize(s), "spadd: sync");
+    }
+    st = launch_partition(A, B, w, true, s);
+    if (st != MSP_OK) return st;
+    st = (A->dtype == MSP_F64) ? launch_tiles<double, ADD_FUSED>(A, B, w, Crp, Ccol, Cval, cap, s)
+                               : launch_tiles<float, ADD_FUSED>(A, B, w, Crp, Ccol, Cval, cap, s);
+    if (st != MSP_OK) return st;
+    // nnz(C) twice: C.row_offsets[m] (from the row ends) and the tiles' total
+    int64_t hbuf[2] = {0, 0};
+    int64_t *pin = pinned_scratch();
+    int64_t *h = pin ? pin : hbuf;
+    h[0] = 0;
+    st = cuda_check(cudaMemcpyAsync(&h[0], Crp + m, sizeof(int32_t), cudaMemcpyDeviceToHost, s), "spadd: nnz");
+    if (st != MSP_OK) return st;
+    st = cuda_check(cudaMemcpyAsync(&h[1], &w.totals[1], sizeof(int64_t), cudaMemcpyDeviceToHost, s), "spadd: nnz");
+    if (st != MSP_OK) return st;
+    st = cuda_check(cudaStreamSynchronize(s), "spadd: sync");
+    if (st != MSP_OK) return st;
+    const int64_t rows_total = int64_t(int32_t(uint32_t(uint64_t(h[0]))));
+    if (h[1] > INT32_MAX) {
+        set_error("spadd: nnz(C) = %lld exceeds int32", (long long)h[1]);
+        return MSP_ERR_OVERFLOW;
+    }
+    if (rows_total != h[1] || h[1] > cap) {
+        set_error("spadd: row total %lld != tile total %lld (unsorted or duplicate columns?)", (long long)rows_total,
+                  (long long)h[1]);
+        return MSP_ERR_INPUT;
+    }
+    *nnzC = h[1];
+    return MSP_OK;
 }
 
 }  // namespace msp

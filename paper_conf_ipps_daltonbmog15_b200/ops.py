@@ -190,6 +190,33 @@ def spadd(A: CsrTensor, B: CsrTensor, stream=None) -> CsrTensor:
     return p.numeric()
 
 
+def spadd_fused(A: CsrTensor, B: CsrTensor, stream=None, col: torch.Tensor | None = None,
+                val: torch.Tensor | None = None) -> CsrTensor:
+    """C = A + B in one pass (msp_spadd_fused; same result as spadd() bit for
+    bit).  col / val, if given, need nnz(A) + nnz(B) entries; the returned
+    C.col / C.vals are views of their first nnz(C) entries."""
+    a, b = A.c(), B.c()
+    if A.shape != B.shape:
+        raise ValueError("A and B differ in shape")
+    dev = A.device
+    cap = A.nnz + B.nnz
+    n = ctypes.c_size_t(0)
+    check("msp_spadd_workspace", lib().msp_spadd_workspace(ctypes.byref(a), ctypes.byref(b), ctypes.byref(n)))
+    ws = workspace(int(n.value), dev, "spadd", stream)
+    _claim(next(_TOKENS), dev, ("spadd",), stream)  # any SpAddPlan's partition in this slot is gone
+    rp = torch.empty(A.shape[0] + 1, dtype=torch.int32, device=dev)
+    col = col if col is not None else torch.empty(max(cap, 1), dtype=torch.int32, device=dev)
+    val = val if val is not None else torch.empty(max(cap, 1), dtype=A.dtype, device=dev)
+    if col.numel() < cap or val.numel() < cap:
+        raise ValueError("col / val need nnz(A) + nnz(B) entries")
+    nnz = ctypes.c_int64(0)
+    check("msp_spadd_fused", lib().msp_spadd_fused(ctypes.byref(a), ctypes.byref(b), rp.data_ptr(), col.data_ptr(),
+                                                   val.data_ptr(), cap, ctypes.byref(nnz), ws.data_ptr(), ws.numel(),
+                                                   _stream_ptr(dev, stream)))
+    k = int(nnz.value)
+    return CsrTensor(rp, col[:k], val[:k], A.shape)
+
+
 # ----------------------------------------------------------------- SpGEMM
 
 class SpGemmPlan:
@@ -356,11 +383,16 @@ _KEY_T = {torch.int32: 4, torch.int64: 8, torch.uint32: 4, torch.uint64: 8}
 
 
 def set_operation(op: str, a_keys: torch.Tensor, b_keys: torch.Tensor, a_vals: torch.Tensor | None = None,
-                  b_vals: torch.Tensor | None = None, stream=None):
+                  b_vals: torch.Tensor | None = None, stream=None, sync: bool = True):
     """Balanced-path set operation on sorted key lists: keys are
     compared as unsigned 32/64-bit integers (int32/int64 tensors are
     reinterpreted), duplicates are key-rank pairs.  Returns (keys, vals or
-    None), trimmed to the result size (msp_set_operation synchronises)."""
+    None), trimmed to the result size (msp_set_operation synchronises).
+
+    sync=False calls msp_set_operation_async instead and returns (keys, vals
+    or None, count): untrimmed output buffers of the result bound and a
+    device int64[2] tensor holding [result size, unsorted-input flag],
+    written in stream order -- no host round trip."""
     code = SET_OPS[op]
     if a_keys.dtype != b_keys.dtype or a_keys.dtype not in _KEY_T:
         raise ValueError("keys must share a 32/64-bit integer dtype")
@@ -382,6 +414,13 @@ def set_operation(op: str, a_keys: torch.Tensor, b_keys: torch.Tensor, a_vals: t
     n = ctypes.c_size_t(0)
     check("msp_set_op_workspace", lib().msp_set_op_workspace(na, nb, ctypes.byref(n)))
     ws = workspace(int(n.value), dev, "setop", stream)
+    if not sync:
+        count = torch.empty(2, dtype=torch.int64, device=dev)
+        check("msp_set_operation_async", lib().msp_set_operation_async(
+            code, a_keys.data_ptr(), a_vals.data_ptr() if vb else None, na, b_keys.data_ptr(),
+            b_vals.data_ptr() if vb else None, nb, kb, vb, ck.data_ptr(), cv.data_ptr() if vb else None, bound,
+            count.data_ptr(), ws.data_ptr(), ws.numel(), _stream_ptr(dev, stream)))
+        return ck, cv, count
     nc = ctypes.c_int64(0)
     check("msp_set_operation", lib().msp_set_operation(
         code, a_keys.data_ptr(), a_vals.data_ptr() if vb else None, na, b_keys.data_ptr(),

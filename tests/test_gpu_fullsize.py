@@ -120,6 +120,10 @@ def test_c3_spadd_full(c3):
     W = oracle.spadd(Ar, T)
     assert np.array_equal(rp, W.rp) and np.array_equal(col, W.col)
     assert np.array_equal(val.view(np.uint32), W.val.view(np.uint32))
+    from paper_conf_ipps_daltonbmog15_b200 import spadd_fused
+    rp, col, val = spadd_fused(dev(Ar), dev(T)).numpy()
+    assert np.array_equal(rp, W.rp) and np.array_equal(col, W.col), "fused: structure"
+    assert np.array_equal(val.view(np.uint32), W.val.view(np.uint32)), "fused: values"
 
 
 def test_c5_spmv_full():

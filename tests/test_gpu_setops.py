@@ -119,3 +119,35 @@ def test_fig2_scale(kind):
         check("union", a, b, np.arange(n, dtype=np.int64), -np.arange(n, dtype=np.int64), label="2e7 pairs-64")
     else:
         check("union", a, b, label="2e7 keys-32")
+
+
+@pytest.mark.parametrize("op", OPS)
+def test_async_form(op):
+    """msp_set_operation_async: same keys / values as the oracle, the size and
+    the unsorted flag land in a device int64[2] in stream order; several
+    calls queued back to back on one stream (shared workspace) without a
+    host sync in between, including an empty one and an unsorted one."""
+    from paper_conf_ipps_daltonbmog15_b200 import set_operation
+    rng = np.random.default_rng(17)
+    cases = []
+    for na, nb, hi in [(30000, 20000, 4000), (0, 0, 10), (1, 3000, 5), (50000, 50000, 10**9)]:
+        a = sorted_keys(rng, na, hi, np.uint32)
+        b = sorted_keys(rng, nb, hi, np.uint32)
+        av = rng.standard_normal(na)
+        bv = rng.standard_normal(nb)
+        cases.append((a, b, av, bv))
+    bad = cases[0][0].copy()
+    bad[100:200] = bad[100:200][::-1]
+    outs = []
+    for a, b, av, bv in cases + [(bad, cases[0][1], cases[0][2], cases[0][3])]:
+        ta = torch.from_numpy(a.view(np.int32)).cuda()
+        tb = torch.from_numpy(b.view(np.int32)).cuda()
+        outs.append(set_operation(op, ta, tb, torch.from_numpy(av).cuda(), torch.from_numpy(bv).cuda(), sync=False))
+    torch.cuda.synchronize()
+    for (a, b, av, bv), (k, v, cnt) in zip(cases, outs):
+        n, flag = cnt.cpu().tolist()
+        ek, ev = oracle.set_op(op, a, b, av, bv)
+        assert flag == 0 and n == ek.size
+        assert np.array_equal(k[:n].cpu().numpy().view(np.uint32), ek)
+        assert np.array_equal(v[:n].cpu().numpy().view(np.uint8), ev.view(np.uint8))
+    assert outs[-1][2][1].item() != 0, "unsorted keys must raise the device flag"

@@ -12,19 +12,23 @@ from tests.gpu_util import dev, tile_edge_matrix
 pytestmark = pytest.mark.gpu
 
 
-def run(A: gen.CSR, B: gen.CSR):
-    from paper_conf_ipps_daltonbmog15_b200 import spadd
-    C = spadd(dev(A), dev(B))
+def run(A: gen.CSR, B: gen.CSR, fused=False):
+    from paper_conf_ipps_daltonbmog15_b200 import spadd, spadd_fused
+    C = (spadd_fused if fused else spadd)(dev(A), dev(B))
     rp, col, val = C.numpy()
     return rp, col, val
 
 
 def check(A, B, label=""):
-    rp, col, val = run(A, B)
+    """Both forms -- two-phase (symbolic + numeric) and the fused
+    one-pass msp_spadd_fused -- against the oracle, bit-exact."""
     W = oracle.spadd(A, B)
-    assert np.array_equal(rp, W.rp), f"{label}: row_offsets differ"
-    assert np.array_equal(col, W.col), f"{label}: col_idx differ"
-    assert np.array_equal(val.view(np.uint8), W.val.view(np.uint8)), f"{label}: values differ"
+    for fused in (False, True):
+        rp, col, val = run(A, B, fused)
+        form = "fused" if fused else "two-phase"
+        assert np.array_equal(rp, W.rp), f"{label} ({form}): row_offsets differ"
+        assert np.array_equal(col, W.col), f"{label} ({form}): col_idx differ"
+        assert np.array_equal(val.view(np.uint8), W.val.view(np.uint8)), f"{label} ({form}): values differ"
 
 
 def test_paper_example(paper_example):
@@ -102,3 +106,45 @@ def test_deterministic():
     r1, c1, v1 = run(A, B)
     r2, c2, v2 = run(A, B)
     assert np.array_equal(v1.view(np.uint8), v2.view(np.uint8))
+
+
+def test_fused_capacity_and_unsorted():
+    """msp_spadd_fused: capacity below nnz(A) + nnz(B) is MSP_ERR_SHAPE; an
+    unsorted row is MSP_ERR_INPUT (row-end and tile totals disagree) or a
+    structure that differs from the oracle's, never an out-of-bounds store."""
+    import torch
+    from paper_conf_ipps_daltonbmog15_b200 import MspError, spadd_fused
+    import ctypes
+    from paper_conf_ipps_daltonbmog15_b200 import lib
+    A = gen.random_csr(400, 300, 3, density=0.05)
+    with pytest.raises(ValueError):   # the binding checks the capacity first
+        spadd_fused(dev(A), dev(A), col=torch.empty(A.nnz, dtype=torch.int32, device="cuda"),
+                    val=torch.empty(A.nnz, dtype=torch.float64, device="cuda"))
+    dA = dev(A)
+    a = dA.c()
+    n = ctypes.c_size_t(0)
+    assert lib().msp_spadd_workspace(ctypes.byref(a), ctypes.byref(a), ctypes.byref(n)) == 0
+    ws = torch.zeros(int(n.value), dtype=torch.uint8, device="cuda")
+    rp = torch.empty(A.m + 1, dtype=torch.int32, device="cuda")
+    c = torch.empty(2 * A.nnz, dtype=torch.int32, device="cuda")
+    v = torch.empty(2 * A.nnz, dtype=torch.float64, device="cuda")
+    nnz = ctypes.c_int64(0)
+    st = lib().msp_spadd_fused(ctypes.byref(a), ctypes.byref(a), rp.data_ptr(), c.data_ptr(), v.data_ptr(),
+                               2 * A.nnz - 1, ctypes.byref(nnz), ws.data_ptr(), ws.numel(), None)
+    assert st == 3  # MSP_ERR_SHAPE: capacity below nnz(A) + nnz(B)
+    st = lib().msp_spadd_fused(ctypes.byref(a), ctypes.byref(a), rp.data_ptr(), c.data_ptr(), v.data_ptr(),
+                               2 * A.nnz, ctypes.byref(nnz), ws.data_ptr(), ws.numel(), None)
+    assert st == 0 and nnz.value == A.nnz
+    bad = A.col.copy()
+    r = int(np.argmax(np.diff(A.rp)))
+    bad[A.rp[r]:A.rp[r + 1]] = bad[A.rp[r]:A.rp[r + 1]][::-1]
+    U = gen.CSR(A.m, A.n, A.rp, bad, A.val)
+    guard = 4096
+    col = torch.full((2 * A.nnz + guard,), -7, dtype=torch.int32, device="cuda")
+    val = torch.zeros(2 * A.nnz + guard, dtype=torch.float64, device="cuda")
+    try:
+        spadd_fused(dev(U), dev(A), col=col[:2 * A.nnz], val=val[:2 * A.nnz])
+    except MspError as err:
+        assert err.status == 6
+    torch.cuda.synchronize()
+    assert (col[2 * A.nnz:] == -7).all(), "store past C_capacity"

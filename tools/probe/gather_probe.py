@@ -23,6 +23,30 @@ idx = torch.empty(4 * m, dtype=torch.int32, device="cuda")
 y = torch.empty(m, dtype=torch.float64, device="cuda")
 names = ["ldg", "ldcg", "nc.L1::no_allocate", "nc.L2::64B", "nc.L2::cache_hint(0)"]
 reps = int(os.environ.get("REPS", "5"))
+if os.environ.get("CSR"):  # the column stream of a BJ config instead of uniform random indices
+    sys.path.insert(0, os.path.dirname(os.path.dirname(_HERE)))
+    import gen
+    A = gen.config(os.environ["CSR"], "int")
+    m = A.nnz // 4
+    idx = torch.as_tensor(A.col[:4 * m], device="cuda")
+    y = torch.empty(m, dtype=torch.float64, device="cuda")
+    x = torch.ones(A.n, dtype=torch.float64, device="cuda")
+    for mode in range(5):
+        for blocks in (148 * 8, 148 * 32):
+            f = lambda: L.probe_gather(mode, ctypes.c_void_p(idx.data_ptr()), ctypes.c_void_p(x.data_ptr()),  # noqa
+                                       ctypes.c_void_p(y.data_ptr()), ctypes.c_longlong(m), blocks, ctypes.c_void_p(s))
+            f()
+            torch.cuda.synchronize()
+            e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+            e0.record()
+            for _ in range(reps):
+                f()
+            e1.record()
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / reps
+            print(json.dumps({"csr": os.environ["CSR"], "nnz": 4 * m, "x_MB": A.n * 8 / 1e6, "mode": names[mode],
+                              "blocks": blocks, "us": round(ms * 1e3, 1)}), flush=True)
+    sys.exit(0)
 for lg in [int(a) for a in sys.argv[1:]] or [20, 23, 26, 27]:
     n = 1 << lg
     x = torch.ones(n, dtype=torch.float64, device="cuda")

@@ -19,11 +19,11 @@ def main():
         x = torch.from_numpy(gen.matrices.x_vector(A.n, "random", dtype=A.val.dtype)).cuda()
         for _ in range(reps):
             msp.spmv(dA, x)
-    elif op == "spadd":
+    elif op in ("spadd", "spadd_fused"):
         T = gen.matrices.transpose(A)
         dT = msp.CsrTensor.from_arrays(T.rp, T.col, T.val, (T.m, T.n), "cuda")
         for _ in range(reps):
-            msp.spadd(dA, dT)
+            (msp.spadd_fused if op == "spadd_fused" else msp.spadd)(dA, dT)
     else:
         for _ in range(reps):
             p = msp.SpGemmPlan(dA, dA)
