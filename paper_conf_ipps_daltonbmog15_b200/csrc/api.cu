@@ -83,7 +83,7 @@ int64_t *pinned_scratch()
 // Large-shared-memory opt-in, once per (device, kernel): the attribute is a
 // per-device property, so a process driving several GPUs sets it on each.
 // Returns the occupancy (resident CTAs per SM) when `threads` > 0.
-msp_status set_smem_attr(const void *func, int smem_bytes, const char *where, int threads, int *occ)
+msp_status set_smem_attr(const void *func, int smem_bytes, const char *where, int threads, int *occ, bool fit_l1)
 {
     struct Entry {
         int dev;
@@ -111,6 +111,30 @@ msp_status set_smem_attr(const void *func, int smem_bytes, const char *where, in
         st = cuda_check(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, func, threads, size_t(smem_bytes)), where);
         if (st != MSP_OK) return st;
         if (o < 1) o = 1;
+        if (fit_l1) {
+            // shrink the carveout to what `o` CTAs need (+1 KB reserved per
+            // CTA): the rest of the SM's 256 KB stays L1, whose lines also
+            // hold the in-flight misses of the gathers
+            int max_smem = 0;
+            if (cudaDeviceGetAttribute(&max_smem, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev) != cudaSuccess ||
+                max_smem <= 0)
+                max_smem = 228 * 1024;
+            const int64_t need = int64_t(o) * (smem_bytes + 1024);
+            int pct = int((need * 100 + max_smem - 1) / max_smem);
+            if (pct < 100) {
+                st = cuda_check(cudaFuncSetAttribute(func, cudaFuncAttributePreferredSharedMemoryCarveout, pct), where);
+                if (st != MSP_OK) return st;
+                int o2 = 0;
+                st = cuda_check(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o2, func, threads, size_t(smem_bytes)),
+                                where);
+                if (st != MSP_OK) return st;
+                if (o2 < o) {  // the driver's carveout steps did not fit: keep the full carveout
+                    st = cuda_check(cudaFuncSetAttribute(func, cudaFuncAttributePreferredSharedMemoryCarveout, 100),
+                                    where);
+                    if (st != MSP_OK) return st;
+                }
+            }
+        }
     }
     if (n < 1024) table[n++] = Entry{dev, func, o};
     if (occ) *occ = o;

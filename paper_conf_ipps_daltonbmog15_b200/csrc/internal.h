@@ -25,7 +25,10 @@ uint64_t launch_count();
 int64_t *pinned_scratch();
 // cudaFuncAttributeMaxDynamicSharedMemorySize (and, with threads > 0, the
 // max carveout + occupancy query) once per (device, kernel).
-msp_status set_smem_attr(const void *func, int smem_bytes, const char *where, int threads = 0, int *occ = nullptr);
+// fit_l1: then shrink the carveout to the occupancy's shared memory, the rest
+// of the SM's unified 256 KB staying L1.
+msp_status set_smem_attr(const void *func, int smem_bytes, const char *where, int threads = 0, int *occ = nullptr,
+                         bool fit_l1 = false);
 
 inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 

@@ -197,6 +197,18 @@ __device__ __forceinline__ T gather_x(const T *p)
     return __ldcg(p);
 #elif MSP_SPMV_GATHER == 2
     return __ldcs(p);
+#elif MSP_SPMV_GATHER == 4
+    T v;
+    if constexpr (sizeof(T) == 8) {
+        double d;
+        asm volatile("ld.global.nc.L2::64B.f64 %0, [%1];" : "=d"(d) : "l"(p));
+        v = T(d);
+    } else {
+        float f;
+        asm volatile("ld.global.nc.L2::64B.f32 %0, [%1];" : "=f"(f) : "l"(p));
+        v = T(f);
+    }
+    return v;
 #elif MSP_SPMV_GATHER == 3
     T v;
     if constexpr (sizeof(T) == 8) {
@@ -914,14 +926,20 @@ template <typename V> struct Shape<V, 3> { using C = Cfg<V, 8, 2, 4, 2>; };
 template <typename V> struct Shape<V, 4> { using C = Cfg<V, 4, 2, 4, 4>; };
 template <typename V> struct Shape<V, 5> { using C = Cfg<V, 4, 2, 4, 5>; };
 template <typename V> struct Shape<V, 6> { using C = Cfg<V, 2, 2, 4, 8>; };
-constexpr int kNumShapes = 7;
+template <typename V> struct Shape<V, 7> { using C = Cfg<V, 2, 2, 4, 6>; };
+constexpr int kNumShapes = 8;
 
 template <typename V, class C>
 msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
 {
     auto kern = spmv_merge_kernel<V, C>;
     int occ = 1;
-    msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), C::SMEM, "spmv: smem", C::THREADS, &occ);
+    // the transpose walk's gathers need L1 lines for their in-flight misses:
+    // carveout fitted to the occupancy (C3 534 -> 454 us, C4 103 -> 83 us,
+    // C5 12.7 -> 9.0 ms; profiles/r2/spmv_irregular_shapes.txt)
+    static const bool fit = !getenv("MSP_SPMV_FULL_CARVEOUT");
+    msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), C::SMEM, "spmv: smem", C::THREADS, &occ,
+                                  fit && !C::ROWK);
     if (st != MSP_OK) return st;
     if (occ > 8) occ = 8;
     static bool said = false;
@@ -1040,6 +1058,7 @@ msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_
     case 4: return launch_cfg<V, typename Shape<V, 4>::C>(A, x, y, ws, ws_bytes, s);
     case 5: return launch_cfg<V, typename Shape<V, 5>::C>(A, x, y, ws, ws_bytes, s);
     case 6: return launch_cfg<V, typename Shape<V, 6>::C>(A, x, y, ws, ws_bytes, s);
+    case 7: return launch_cfg<V, typename Shape<V, 7>::C>(A, x, y, ws, ws_bytes, s);
     default: return launch_cfg<V, typename Shape<V, 0>::C>(A, x, y, ws, ws_bytes, s);
     }
 }

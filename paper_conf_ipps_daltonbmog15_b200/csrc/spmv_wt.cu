@@ -521,7 +521,8 @@ msp_status launch_wt(const msp_csr *A, const void *x, void *y, void *ws, size_t 
     using C = WtCfg<V, K, 11, (NSUB0 < 24 ? NSUB0 : 24), 3>;
     auto kern = spmv_wt_kernel<V, C>;
     int occ = 1;
-    msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), C::SMEM, "spmv_wt: smem", C::THREADS, &occ);
+    static const bool fit = getenv("MSP_SPMV_WT_L1") != nullptr;  // experiment: carveout fitted to the CTA
+    msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), C::SMEM, "spmv_wt: smem", C::THREADS, &occ, fit);
     if (st != MSP_OK) return st;
     static bool said = false;
     if (!said && getenv("MSP_VERBOSE")) {

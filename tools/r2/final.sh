@@ -16,3 +16,4 @@ done
 python tools/dense_spgemm.py 1000 2000 > $D/dense.txt 2>&1
 MSP_SPGEMM_SEGMENTED=0 python tools/dense_spgemm.py 1000 > $D/dense_esc.txt 2>&1
 for c in C1 C2 C3 C4 C5; do python tools/spmv_tune.py $c "VERBOSE=1" >> $D/spmv_default_tune.txt 2>&1; done
+timeout 600 python tools/setops_bench.py > $D/setops.txt 2>&1; echo setops $?

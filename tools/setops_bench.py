@@ -44,10 +44,10 @@ def main():
                     res = call()
                 torch.cuda.synchronize()
                 if mode == "graph":  # the async call captured once, replayed: no host work per call
-                    g = torch.cuda.CUDAGraph()
-                    with torch.cuda.graph(g):
-                        res = call()
-                    call = g.replay
+                    graph = torch.cuda.CUDAGraph()
+                    with torch.cuda.graph(graph):
+                        cres = call()
+                    call = graph.replay
                     for _ in range(3):
                         call()
                     torch.cuda.synchronize()
@@ -60,6 +60,8 @@ def main():
                 e1.record()
                 torch.cuda.synchronize()
                 ms = e0.elapsed_time(e1) / reps
+                if mode == "graph":
+                    res = cres
                 nout = res[0].numel() if mode == "sync" else int(res[2][0].item())
                 w = a.element_size() + (av.element_size() if av is not None else 0)
                 by = (2 * n + nout) * w
