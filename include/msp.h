@@ -64,7 +64,7 @@
 extern "C" {
 #endif
 
-#define MSP_VERSION 4  /* 2: msp_spgemm_info passed to symbolic / numeric; 3: segmented_rows; 4: msp_set_operation_async, msp_spadd_fused */
+#define MSP_VERSION 5  /* 2: msp_spgemm_info passed to symbolic / numeric; 3: segmented_rows; 4: msp_set_operation_async, msp_spadd_fused; 5: row_accumulator */
 
 typedef enum {
     MSP_OK = 0,
@@ -216,6 +216,15 @@ typedef struct {
                                 pass: output span <= 12288 columns and >= 1
                                 product per 4 columns of it (
                                 MSP_SPGEMM_SEGMENTED=0 disables) */
+    int64_t row_accumulator; /* 1: every short row's output span is at most
+                                65,536 columns, so the short rows take the
+                                row-accumulator path (a warp per row: bitmap
+                                count in symbolic, shared-memory accumulation
+                                in k order in numeric) and no product tile
+                                runs; 0: the ESC tile pass.  main_ws then holds
+                                one int32 per product (each short row's column
+                                list) instead of the tile permutations.
+                                MSP_SPGEMM_ROWACC=0 disables (ablation). */
 } msp_spgemm_info;
 
 msp_status msp_spgemm_setup_workspace(const msp_csr *A, const msp_csr *B, size_t *bytes);

@@ -127,7 +127,7 @@ struct AddLayout {
     // the output run overlays the input windows: it is written only after
     // the scan barrier, when every thread has finished reading them
     static constexpr int O_OFF = 0;
-    static_assert(OBYTES <= V_OFF + VBYTES, "output run must fit over the input windows");
+    static_assert(O_OFF + OBYTES <= V_OFF + VBYTES, "output run must fit over the input windows");
     static constexpr int ST_OFF = (V_OFF + VBYTES + 15) / 16 * 16;
     static constexpr int WS_OFF = ST_OFF + int(sizeof(Split)) * (ADD_NT + 1);
     static constexpr int BAR_OFF = (WS_OFF + 4 * (ADD_NT / 32) + 15) / 16 * 16;

@@ -276,6 +276,251 @@ spa_row_kernel(const int32_t *__restrict__ sparow, const int32_t *__restrict__ A
     }
 }
 
+// ------------------------------------------ row accumulator for short rows
+// The same idea as the segmented path, for SHORT rows (a B200 addition in
+// the direction of the paper's future work): when every short
+// row's output columns span at most WR_SPAN columns, the whole short-row
+// product set skips expansion + sort.  One warp owns one row:
+//   symbolic: marks the row's output columns in a warp-private bitmap over
+//             its span, counts them and writes them ascending into a
+//             scratch list at the row's product offset S[rp[r]] (at most P_r
+//             entries);
+//   numeric:  reads that list (ranks by binary search in shared memory),
+//             zero-free accumulates a_ik * b_kj into a shared-memory
+//             accumulator for k in A's column order (one k per step, a
+//             __syncwarp between steps: a B row has distinct columns, so the
+//             lanes of a step never collide), and writes the row of C.
+// Every column sums its products in Gustavson's order with separate multiply
+// and add roundings, as the oracle does.  The choice is global (all short
+// rows or none) so that the tile pass is either skipped or untouched.
+constexpr int WR_SPAN = 65536;            // bitmap bits per warp (8 KB)
+constexpr int WR_WORDS = WR_SPAN / 32;
+constexpr int WR_SYM_WARPS = 8;           // 64 KB of bitmaps per CTA
+constexpr int WR_UMAX = 512;              // accumulator entries per warp per pass (6 KB with the column list)
+constexpr int WR_NUM_WARPS = 8;
+
+__device__ __forceinline__ int warp_excl_sum(int v, int lane, int *total)
+{
+    const int inc = warp_inclusive_sum(v, lane);
+    *total = __shfl_sync(0xffffffffu, inc, 31);
+    return inc - v;
+}
+
+// Span of every short row with products (warp per row); counts the short
+// rows whose span exceeds WR_SPAN into *fail.
+__global__ void wr_span_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
+                               const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
+                               const uint8_t *__restrict__ rowlong, int32_t *__restrict__ lo_out,
+                               int32_t *__restrict__ hi_out, unsigned long long *__restrict__ fail)
+{
+    const int lane = threadIdx.x & 31;
+    const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
+    unsigned long long nfail = 0;
+    for (int64_t r = int64_t(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5); r < m; r += nwarps) {
+        if (rowlong[r]) continue;
+        const int32_t a0 = Arp[r], a1 = Arp[r + 1];
+        int32_t lo = INT_MAX, hi = -1;
+        for (int32_t j = a0 + lane; j < a1; j += 32) {
+            const int32_t k = Acol[j], b0 = Brp[k], b1 = Brp[k + 1];
+            if (b1 > b0) {
+                lo = min(lo, Bcol[b0]);
+                hi = max(hi, Bcol[b1 - 1]);
+            }
+        }
+        lo = __reduce_min_sync(0xffffffffu, lo);
+        hi = __reduce_max_sync(0xffffffffu, hi);
+        if (lane == 0) {
+            lo_out[r] = lo;
+            hi_out[r] = hi;
+            if (hi >= lo && int64_t(hi) - lo + 1 > WR_SPAN) ++nfail;
+        }
+    }
+    if (lane == 0 && nfail) atomicAdd(fail, nfail);
+}
+
+// Symbolic: bitmap mark, count, ascending column list at ucol + S[rp[r]].
+__global__ void __launch_bounds__(WR_SYM_WARPS * 32)
+wr_symbolic_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
+                   const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
+                   const uint8_t *__restrict__ rowlong, const int64_t *__restrict__ S,
+                   const int32_t *__restrict__ spanlo, const int32_t *__restrict__ spanhi,
+                   int32_t *__restrict__ Crp_counts, int32_t *__restrict__ ucol)
+{
+    extern __shared__ __align__(16) uint32_t wr_bm_all[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint32_t *bm = wr_bm_all + warp * WR_WORDS;
+    const int64_t nwarps = int64_t(gridDim.x) * WR_SYM_WARPS;
+    for (int64_t r = int64_t(blockIdx.x) * WR_SYM_WARPS + warp; r < m; r += nwarps) {
+        if (rowlong[r]) continue;
+        const int32_t lo = spanlo[r], hi = spanhi[r];
+        if (hi < lo) {  // no products
+            if (lane == 0) Crp_counts[r] = 0;
+            continue;
+        }
+        const int nw = (hi - lo + 32) >> 5;
+        for (int w = lane; w < nw; w += 32) bm[w] = 0u;
+        __syncwarp();
+        const int32_t a0 = Arp[r], a1 = Arp[r + 1];
+        for (int32_t jc = a0; jc < a1; jc += 32) {
+            const int32_t j = jc + lane;
+            const int nl = min(32, a1 - jc);
+            int32_t b0 = 0, len = 0;
+            if (j < a1) {
+                const int32_t k = Acol[j];
+                b0 = Brp[k];
+                len = Brp[k + 1] - b0;
+            }
+            int tot;
+            const int off = warp_excl_sum(len, lane, &tot);
+            // products of the chunk, flattened over the lanes, 8 loads in flight per lane
+            for (int t0 = 0; t0 < tot; t0 += 32 * 8) {
+                int32_t c[8];
+#pragma unroll
+                for (int u = 0; u < 8; ++u) {
+                    const int t = t0 + u * 32 + lane;
+                    int sidx = 0;  // lane owning product t: the last lane with off <= t
+#pragma unroll
+                    for (int step = 16; step >= 1; step >>= 1) {
+                        const int cand = sidx + step;
+                        const int oc = __shfl_sync(0xffffffffu, off, cand & 31);
+                        if (cand < nl && oc <= t) sidx = cand;
+                    }
+                    const int ob = __shfl_sync(0xffffffffu, off, sidx);
+                    const int32_t bb = __shfl_sync(0xffffffffu, b0, sidx);
+                    c[u] = t < tot ? Bcol[bb + (t - ob)] : -1;
+                }
+#pragma unroll
+                for (int u = 0; u < 8; ++u)
+                    if (c[u] >= 0) {
+                        const int x = c[u] - lo;
+                        atomicOr(&bm[x >> 5], 1u << (x & 31));
+                    }
+            }
+        }
+        __syncwarp();
+        int cnt = 0;
+        for (int w = lane; w < nw; w += 32) cnt += __popc(bm[w]);
+        cnt = __reduce_add_sync(0xffffffffu, cnt);
+        if (lane == 0) Crp_counts[r] = cnt;
+        // ascending column list at the row's product offset
+        int32_t *dst = ucol + S[a0];
+        int run = 0;
+        for (int w0 = 0; w0 < nw; w0 += 32) {
+            const int w = w0 + lane;
+            uint32_t word = w < nw ? bm[w] : 0u;
+            int wt;
+            int p = run + warp_excl_sum(__popc(word), lane, &wt);
+            while (word) {
+                const int b = __ffs(word) - 1;
+                word &= word - 1;
+                dst[p++] = lo + w * 32 + b;
+            }
+            run += wt;
+        }
+        __syncwarp();  // the bitmap is reused by the warp's next row
+    }
+}
+
+// Numeric: accumulate into shared memory in k order, WR_UMAX columns per pass.
+template <typename V>
+__global__ void __launch_bounds__(WR_NUM_WARPS * 32)
+wr_numeric_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
+                  const V *__restrict__ Aval, const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
+                  const V *__restrict__ Bval, const uint8_t *__restrict__ rowlong, const int64_t *__restrict__ S,
+                  const int32_t *__restrict__ ucol, const int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol,
+                  V *__restrict__ Cval)
+{
+    __shared__ int32_t s_uc[WR_NUM_WARPS][WR_UMAX];
+    __shared__ double s_acc[WR_NUM_WARPS][WR_UMAX];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    int32_t *uc = s_uc[warp];
+    double *acc = s_acc[warp];
+    const int64_t nwarps = int64_t(gridDim.x) * WR_NUM_WARPS;
+    for (int64_t r = int64_t(blockIdx.x) * WR_NUM_WARPS + warp; r < m; r += nwarps) {
+        if (rowlong[r]) continue;
+        const int32_t cb = Crp[r], U = Crp[r + 1] - cb;
+        if (U == 0) continue;
+        const int32_t a0 = Arp[r], a1 = Arp[r + 1];
+        const int32_t *src = ucol + S[a0];
+        for (int cs = 0; cs < U; cs += WR_UMAX) {
+            const int nu = min(WR_UMAX, U - cs);
+            for (int i = lane; i < nu; i += 32) {
+                uc[i] = src[cs + i];
+                acc[i] = -0.0;  // -0 + p == p for every p: the first product needs no special case
+            }
+            __syncwarp();
+            const int32_t cmin = uc[0], cmax = uc[nu - 1];
+            for (int32_t jc = a0; jc < a1; jc += 32) {
+                const int32_t j = jc + lane;
+                const int nl = min(32, a1 - jc);
+                int32_t b0 = 0, len = 0;
+                double av = 0.0;
+                if (j < a1) {
+                    const int32_t k = Acol[j];
+                    b0 = Brp[k];
+                    len = Brp[k + 1] - b0;
+                    av = double(Aval[j]);
+                }
+                if (__all_sync(0xffffffffu, len <= 32)) {
+                    // one B row per step, lane q holds its q-th entry; 8 steps of loads in flight
+                    for (int s0 = 0; s0 < nl; s0 += 8) {
+                        int32_t c[8];
+                        V v[8];
+#pragma unroll
+                        for (int u = 0; u < 8; ++u) {
+                            const int sidx = s0 + u;
+                            const int32_t bb = __shfl_sync(0xffffffffu, b0, sidx & 31);
+                            const int32_t ll = __shfl_sync(0xffffffffu, len, sidx & 31);
+                            const bool ok = sidx < nl && lane < ll;
+                            c[u] = ok ? Bcol[bb + lane] : -1;
+                            v[u] = ok ? Bval[bb + lane] : V(0);
+                        }
+#pragma unroll
+                        for (int u = 0; u < 8; ++u) {
+                            const double a = __shfl_sync(0xffffffffu, av, (s0 + u) & 31);
+                            if (c[u] >= cmin && c[u] <= cmax) {
+                                int lo = 0, hi = nu - 1;  // rank of c in the column list
+                                while (lo < hi) {
+                                    const int mid = (lo + hi) >> 1;
+                                    if (uc[mid] < c[u]) lo = mid + 1;
+                                    else hi = mid;
+                                }
+                                acc[lo] = __dadd_rn(acc[lo], __dmul_rn(a, double(v[u])));
+                            }
+                            __syncwarp();  // the next k's sums follow this one's
+                        }
+                    }
+                } else {
+                    for (int sidx = 0; sidx < nl; ++sidx) {
+                        const int32_t bb = __shfl_sync(0xffffffffu, b0, sidx);
+                        const int32_t ll = __shfl_sync(0xffffffffu, len, sidx);
+                        const double a = __shfl_sync(0xffffffffu, av, sidx);
+                        for (int q = lane; q < ll; q += 32) {
+                            const int32_t c = Bcol[bb + q];
+                            if (c >= cmin && c <= cmax) {
+                                int lo = 0, hi = nu - 1;
+                                while (lo < hi) {
+                                    const int mid = (lo + hi) >> 1;
+                                    if (uc[mid] < c) lo = mid + 1;
+                                    else hi = mid;
+                                }
+                                acc[lo] = __dadd_rn(acc[lo], __dmul_rn(a, double(Bval[bb + q])));
+                            }
+                        }
+                        __syncwarp();
+                    }
+                }
+            }
+            __syncwarp();
+            for (int i = lane; i < nu; i += 32) {
+                Ccol[cb + cs + i] = uc[i];
+                Cval[cb + cs + i] = V(acc[i]);
+            }
+            __syncwarp();
+        }
+    }
+}
+
 struct SetupWs {
     int32_t *arow;
     int64_t *S;          // [nnzA + 1]
@@ -935,6 +1180,7 @@ __global__ void long_emit_kernel(int64_t LP, int64_t nlong, const int64_t *__res
 struct MainWs {
     GSplit *splits;
     uint16_t *perm;  // per tile: the symbolic sort's permutation (GM_T entries)
+    int32_t *ucol;   // row-accumulator path: each short row's output columns at its product offset
     int32_t *Xc[2];
     double *Xv[2];
     int32_t *heads;
@@ -945,12 +1191,13 @@ struct MainWs {
     size_t bytes;
 };
 
-MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, void *ws, size_t cap, bool *ok)
+MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, int64_t nucol, void *ws, size_t cap, bool *ok)
 {
     MainWs w;
     Carve cv(ws, cap);
     w.splits = cv.take<GSplit>(size_t(ntiles + 1));
     w.perm = cv.take<uint16_t>(size_t(ntiles) * GM_T);
+    w.ucol = cv.take<int32_t>(size_t(nucol > 0 ? nucol : 1));
     for (int i = 0; i < 2; ++i) {
         w.Xc[i] = cv.take<int32_t>(size_t(LP > 0 ? LP : 1));
         w.Xv[i] = cv.take<double>(size_t(LP > 0 ? LP : 1));
@@ -966,7 +1213,7 @@ MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, void *ws, size_t cap, b
 }
 
 struct HostInfo {  // read back by setup (one synchronisation), passed to symbolic / numeric in msp_spgemm_info
-    int64_t nprods, nlong, LP, LC, maxP, nspa;
+    int64_t nprods, nlong, LP, LC, maxP, nspa, rowacc;
 };
 
 // The setup sizes gathered into one device array (so setup reads them back
@@ -985,6 +1232,7 @@ __global__ void info_gather_kernel(const int64_t *__restrict__ S, int64_t nnzA, 
     out[3] = nlong > 0 ? longCO[nlong] : 0;
     out[4] = int64_t(stats[0]);
     out[5] = spapos[m];
+    // out[6] is stats[7] itself: short rows whose span is too wide for the row accumulator
 }
 
 // A pinned host staging word array per host thread for the synchronising reads.
@@ -1005,14 +1253,16 @@ msp_status read_back(const int64_t *dev, int n, int64_t *host, cudaStream_t s, c
     return st;
 }
 
+bool rowacc_enabled();
+
 msp_status read_info(const SetupWs &sw, int64_t m, int64_t nnzA, HostInfo *h, cudaStream_t s)
 {
     info_gather_kernel<<<1, 32, 0, s>>>(sw.S, nnzA, sw.longpos, m, sw.longO, sw.longCO, sw.stats, sw.spapos,
                                         reinterpret_cast<int64_t *>(sw.stats) + 1);
     msp_status st = last_launch("info_gather_kernel");
     if (st != MSP_OK) return st;
-    int64_t v[6];
-    st = read_back(reinterpret_cast<const int64_t *>(sw.stats) + 1, 6, v, s, "spgemm: setup sizes");
+    int64_t v[7];
+    st = read_back(reinterpret_cast<const int64_t *>(sw.stats) + 1, 7, v, s, "spgemm: setup sizes");
     if (st != MSP_OK) return st;
     h->nprods = v[0];
     h->nlong = v[1];
@@ -1020,6 +1270,7 @@ msp_status read_info(const SetupWs &sw, int64_t m, int64_t nnzA, HostInfo *h, cu
     h->LC = v[3];
     h->maxP = v[4];
     h->nspa = v[5];
+    h->rowacc = (rowacc_enabled() && v[6] == 0) ? 1 : 0;
     return MSP_OK;
 }
 
@@ -1029,7 +1280,10 @@ msp_status launch_tiles(const msp_csr *A, const msp_csr *B, const SetupWs &sw, c
 {
     auto kern = gemm_tile_kernel<KT, V, NUM>;
     const int smem = int(sizeof(TileSmem<KT, NUM>));
-    msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), smem, "spgemm: tile smem");
+    static const bool fit = getenv("MSP_SPGEMM_FIT") != nullptr;  // experiment: carveout fitted to the CTAs
+    msp_status st = fit ? set_smem_attr(reinterpret_cast<const void *>(kern), smem, "spgemm: tile smem", GM_NT,
+                                        nullptr, true)
+                        : set_smem_attr(reinterpret_cast<const void *>(kern), smem, "spgemm: tile smem");
     if (st != MSP_OK) return st;
     kern<<<unsigned(ntiles), GM_NT, smem, s>>>(A->col_idx, static_cast<const V *>(A->vals), B->row_offsets,
                                                 B->col_idx, static_cast<const V *>(B->vals), sw.arow, sw.S,
@@ -1091,6 +1345,57 @@ msp_status run_long(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const
     return last_launch("long_emit_kernel");
 }
 
+bool rowacc_enabled()
+{
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("MSP_SPGEMM_ROWACC");  // 0 disables the short-row accumulator (ablation)
+        v = (e && atoi(e) == 0) ? 0 : 1;
+    }
+    return v != 0;
+}
+
+template <bool NUM>
+msp_status run_rowacc(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, int32_t *Crp,
+                      int32_t *Ccol, void *Cval, cudaStream_t s)
+{
+    const int32_t m = A->nrows;
+    if (!NUM) {
+        const int smem = WR_SYM_WARPS * WR_WORDS * 4;
+        int occ = 1;
+        msp_status st = set_smem_attr(reinterpret_cast<const void *>(wr_symbolic_kernel), smem,
+                                      "spgemm: row accumulator smem", WR_SYM_WARPS * 32, &occ, true);
+        if (st != MSP_OK) return st;
+        const int64_t g = std::min<int64_t>(int64_t(occ) * sm_count(), ceil_div(m, WR_SYM_WARPS));
+        wr_symbolic_kernel<<<unsigned(g > 0 ? g : 1), WR_SYM_WARPS * 32, smem, s>>>(
+            m, A->row_offsets, A->col_idx, B->row_offsets, B->col_idx, sw.rowlong, sw.S, sw.spanlo, sw.spanhi,
+            Crp + 1, mw.ucol);
+        return last_launch("wr_symbolic_kernel");
+    }
+    if (A->dtype == MSP_F64) {
+        auto kern = wr_numeric_kernel<double>;
+        int occ = 1;
+        msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), 0, "spgemm: row accumulator",
+                                      WR_NUM_WARPS * 32, &occ, true);
+        if (st != MSP_OK) return st;
+        const int64_t g = std::min<int64_t>(int64_t(occ) * sm_count(), ceil_div(m, WR_NUM_WARPS));
+        kern<<<unsigned(g > 0 ? g : 1), WR_NUM_WARPS * 32, 0, s>>>(
+            m, A->row_offsets, A->col_idx, static_cast<const double *>(A->vals), B->row_offsets, B->col_idx,
+            static_cast<const double *>(B->vals), sw.rowlong, sw.S, mw.ucol, Crp, Ccol, static_cast<double *>(Cval));
+    } else {
+        auto kern = wr_numeric_kernel<float>;
+        int occ = 1;
+        msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), 0, "spgemm: row accumulator",
+                                      WR_NUM_WARPS * 32, &occ, true);
+        if (st != MSP_OK) return st;
+        const int64_t g = std::min<int64_t>(int64_t(occ) * sm_count(), ceil_div(m, WR_NUM_WARPS));
+        kern<<<unsigned(g > 0 ? g : 1), WR_NUM_WARPS * 32, 0, s>>>(
+            m, A->row_offsets, A->col_idx, static_cast<const float *>(A->vals), B->row_offsets, B->col_idx,
+            static_cast<const float *>(B->vals), sw.rowlong, sw.S, mw.ucol, Crp, Ccol, static_cast<float *>(Cval));
+    }
+    return last_launch("wr_numeric_kernel");
+}
+
 bool spa_enabled()
 {
     static int v = -1;
@@ -1117,7 +1422,12 @@ msp_status run_spa(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const 
     return last_launch(NUM ? "spa_row_kernel<numeric>" : "spa_row_kernel<symbolic>");
 }
 
-int64_t ntiles_of(int64_t nnzA, int64_t nprods) { return ceil_div(nnzA + nprods > 0 ? nnzA + nprods : 1, GM_TP); }
+// Product tiles of the main pass (none when the row accumulator takes every short row).
+int64_t ntiles_of(int64_t nnzA, int64_t nprods, int64_t rowacc = 0)
+{
+    if (rowacc) return 0;
+    return ceil_div(nnzA + nprods > 0 ? nnzA + nprods : 1, GM_TP);
+}
 
 msp_status prepare_main(const msp_csr *A, const void *ws1, size_t b1, void *ws2, size_t b2, SetupWs *sw, MainWs *mw,
                         const HostInfo &h)
@@ -1125,7 +1435,7 @@ msp_status prepare_main(const msp_csr *A, const void *ws1, size_t b1, void *ws2,
     bool ok1, ok2;
     *sw = carve_setup(A, const_cast<void *>(ws1), b1, &ok1);
     if (!ok1) return MSP_ERR_WORKSPACE;
-    *mw = carve_main(A->nrows, ntiles_of(A->nnz, h.nprods), h.LP, ws2, b2, &ok2);
+    *mw = carve_main(A->nrows, ntiles_of(A->nnz, h.nprods, h.rowacc), h.LP, h.rowacc ? h.nprods : 0, ws2, b2, &ok2);
     if (!ok2) return MSP_ERR_WORKSPACE;
     return MSP_OK;
 }
@@ -1139,6 +1449,7 @@ HostInfo host_info(const msp_spgemm_info *info)
     h.LC = info->long_chunks;
     h.maxP = info->max_row_products;
     h.nspa = info->segmented_rows;
+    h.rowacc = info->row_accumulator;
     return h;
 }
 
@@ -1194,6 +1505,13 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
             st = last_launch("span_kernel");
             if (st != MSP_OK) return st;
         }
+        if (nnz > 0 && rowacc_enabled()) {  // short-row spans for the row accumulator
+            wr_span_kernel<<<unsigned(std::min<int64_t>(ceil_div(m, 8), 148 * 16)), 256, 0, s>>>(
+                A->nrows, A->row_offsets, A->col_idx, B->row_offsets, B->col_idx, w.rowlong, w.spanlo, w.spanhi,
+                &w.stats[7]);
+            st = last_launch("wr_span_kernel");
+            if (st != MSP_OK) return st;
+        }
         spa_classify_kernel<<<blocks, 256, 0, s>>>(A->nrows, A->row_offsets, w.S, w.spanlo, w.spanhi, w.rowlong,
                                                    w.longflag, w.spaflag);
         st = last_launch("spa_classify_kernel");
@@ -1223,9 +1541,9 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
     HostInfo h;
     st = read_info(w, m, nnz, &h, s);
     if (st != MSP_OK) return st;
-    const int64_t ntiles = ntiles_of(nnz, h.nprods);
+    const int64_t ntiles = ntiles_of(nnz, h.nprods, h.rowacc);
     bool ok2;
-    MainWs mw = carve_main(m, ntiles, h.LP, nullptr, SIZE_MAX, &ok2);
+    MainWs mw = carve_main(m, ntiles, h.LP, h.rowacc ? h.nprods : 0, nullptr, SIZE_MAX, &ok2);
     info->nprods = h.nprods;
     info->ntiles = ntiles;
     info->long_rows = h.nlong;
@@ -1235,6 +1553,7 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
     info->long_chunks = h.LC;
     info->max_tile_span = -1;  // set by symbolic
     info->segmented_rows = h.nspa;
+    info->row_accumulator = h.rowacc;
     return MSP_OK;
 }
 
@@ -1253,9 +1572,14 @@ msp_status spgemm_pass(const msp_csr *A, const msp_csr *B, const void *ws1, size
     msp_status st = prepare_main(A, ws1, b1, ws2, b2, &sw, &mw, h);
     if (st != MSP_OK) return st;
     const int64_t m = A->nrows;
-    const int64_t ntiles = ntiles_of(A->nnz, h.nprods);
+    const int64_t ntiles = ntiles_of(A->nnz, h.nprods, h.rowacc);
     int64_t maxspan = info->max_tile_span;
-    if (!NUM) {
+    if (!NUM && h.rowacc && m > 0) {
+        st = cuda_check(cudaMemsetAsync(Crp, 0, size_t(m + 1) * sizeof(int32_t), s), "spgemm: clear rp");
+        if (st != MSP_OK) return st;
+        maxspan = 0;  // no product tiles
+        info->max_tile_span = 0;
+    } else if (!NUM) {
         st = cuda_check(cudaMemsetAsync(Crp, 0, size_t(m + 1) * sizeof(int32_t), s), "spgemm: clear rp");
         if (st != MSP_OK) return st;
         if (m == 0) {
@@ -1282,9 +1606,11 @@ msp_status spgemm_pass(const msp_csr *A, const msp_csr *B, const void *ws1, size
         set_error("spgemm: numeric needs the info returned by symbolic (max_tile_span unset)");
         return MSP_ERR_ARG;
     }
-    if (h.nprods > 0) {
-        st = (A->dtype == MSP_F64) ? run_tiles<double, NUM>(A, B, sw, mw, ntiles, maxspan, Crp, Ccol, Cval, s)
-                                   : run_tiles<float, NUM>(A, B, sw, mw, ntiles, maxspan, Crp, Ccol, Cval, s);
+    if (h.nprods > 0 && m > 0) {
+        if (h.rowacc) st = run_rowacc<NUM>(A, B, sw, mw, Crp, Ccol, Cval, s);
+        else
+            st = (A->dtype == MSP_F64) ? run_tiles<double, NUM>(A, B, sw, mw, ntiles, maxspan, Crp, Ccol, Cval, s)
+                                       : run_tiles<float, NUM>(A, B, sw, mw, ntiles, maxspan, Crp, Ccol, Cval, s);
         if (st != MSP_OK) return st;
         st = (A->dtype == MSP_F64) ? run_long<double, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s)
                                    : run_long<float, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s);

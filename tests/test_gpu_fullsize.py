@@ -53,6 +53,7 @@ def test_c2_spgemm_full_complete():
     A = gen.config("C2", "random")
     info = assert_spgemm_complete(A, A, "C2 A*A")
     assert info.nprods == 890 ** 3
+    assert info.row_accumulator == 1  # stencil rows: the short-row accumulator path
 
 
 def test_c4_spgemm_full_complete():
@@ -60,6 +61,7 @@ def test_c4_spgemm_full_complete():
     A = gen.config("C4", "int")
     info = assert_spgemm_complete(A, A, "C4 A*A", exact=True)
     assert info.long_rows >= 1
+    assert info.row_accumulator == 0  # uniform rows span ~2e6 columns: ESC tiles
 
 
 def test_spgemm_64bit_keys():

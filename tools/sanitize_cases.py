@@ -1,8 +1,9 @@
 """Small invocations of every libmsp kernel for compute-sanitizer
 (memcheck / racecheck / synccheck): SpMV (warp-tile kernel on a 27-point
 stencil, CTA-tile transpose walk on irregular rows, empty rows, a long row),
-SpAdd, SpGEMM (short and long rows, 32- and 64-bit keys), set operations
-(keys / pairs, all four ops), csr_check and the row-offset rebase.
+SpAdd (two-phase and one-pass), SpGEMM (short and long rows, 32- and 64-bit
+keys, the short-row accumulator), set operations (keys / pairs, all four
+ops, the async form), csr_check and the row-offset rebase.
 Run: compute-sanitizer --tool memcheck python tools/sanitize_cases.py"""
 import sys
 
@@ -30,6 +31,7 @@ def main():
         msp.spmv(dA, x)
         T = gen.transpose(A)
         msp.spadd(dA, dev(T))
+        msp.spadd_fused(dA, dev(T))
         if A.m == A.n and A.nnz < 200_000:
             msp.spgemm(dA, dA)
         msp.csr_check(dA)
@@ -45,6 +47,16 @@ def main():
     bcol = np.concatenate([np.sort(rng.choice(n, size=int(L), replace=False)) for L in bl]).astype(np.int32)
     B = gen.CSR(k, n, brp, bcol, gen.matrices.random_values(bcol.size, 3))
     msp.spgemm(dev(A), dev(B))
+    # SpGEMM row accumulator with > 512 output columns per row (several passes), B rows > 32
+    bl = np.where(rng.random(300) < 0.1, 0, rng.integers(1, 70, 300))
+    brp = np.concatenate([[0], np.cumsum(bl)]).astype(np.int32)
+    bcol = np.concatenate([np.sort(rng.choice(60_000, size=int(L), replace=False)) for L in bl]).astype(np.int32)
+    B = gen.CSR(300, 60_000, brp, bcol, gen.matrices.random_values(bcol.size, 4))
+    al = rng.integers(1, 30, 200)
+    arp = np.concatenate([[0], np.cumsum(al)]).astype(np.int32)
+    acol = np.concatenate([np.sort(rng.choice(300, size=int(L), replace=False)) for L in al]).astype(np.int32)
+    A = gen.CSR(200, 300, arp, acol, gen.matrices.random_values(acol.size, 5))
+    msp.spgemm(dev(A), dev(B))
     # set operations
     a = np.sort(rng.integers(0, 500, 20000)).astype(np.int32)
     b = np.sort(rng.integers(0, 500, 15000)).astype(np.int32)
@@ -52,6 +64,7 @@ def main():
         msp.set_operation(op, torch.from_numpy(a).cuda(), torch.from_numpy(b).cuda())
         msp.set_operation(op, torch.from_numpy(a.astype(np.int64)).cuda(), torch.from_numpy(b.astype(np.int64)).cuda(),
                           torch.from_numpy(a.astype(np.float64)).cuda(), torch.from_numpy(b.astype(np.float64)).cuda())
+        msp.set_operation(op, torch.from_numpy(a).cuda(), torch.from_numpy(b).cuda(), sync=False)
     msp.rebase_offsets(torch.arange(10, dtype=torch.int32, device="cuda"), 5)
     torch.cuda.synchronize()
     print("sanitize cases done", msp.lib().msp_launch_count(), "launches")
