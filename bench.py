@@ -132,8 +132,15 @@ def spadd_alg_bytes(m, nnz_a, nnz_b, nnz_c, vsize):
     return (nnz_a + nnz_b) * (4 + vsize) + nnz_c * (4 + vsize) + 3 * 4 * (m + 1)
 
 
-def spgemm_pass_bytes(m, nnz_a, nprods, nnz_c, vsize):
-    """The ESC method's own traffic per pass:
+def spgemm_pass_bytes(m, nnz_a, nprods, nnz_c, vsize, rowacc=False):
+    """The method's own traffic per pass.  Row accumulator
+    (rowacc): setup as below plus the span pass (A columns, 8 of B offsets
+    and 8 of B columns per A nonzero); symbolic reads A columns and B offsets
+    (12 per A nonzero), gathers one B column per product (4) and writes each
+    row's column list (4 per C nonzero); numeric reads the same plus A values
+    (12 + s per A nonzero), gathers a B column + value per product (4 + s),
+    reads the column list (4 per C nonzero) and writes C (4 + s).
+    ESC:
     setup    -- A offsets + columns read, B offsets gathered (8 per A
                 nonzero), S written (8), COO rows written (4);
     symbolic -- A columns, COO rows and S read (16 per A nonzero), one B
@@ -143,6 +150,11 @@ def spgemm_pass_bytes(m, nnz_a, nprods, nnz_c, vsize):
                 one B column + value gathered per product (4 + s), the
                 permutation read (2), C columns + values written (4 + s)."""
     setup = 4 * (m + 1) + nnz_a * (4 + 8 + 8 + 4)
+    if rowacc:
+        setup += 4 * (m + 1) + nnz_a * (4 + 8 + 8)
+        symbolic = nnz_a * 12 + nprods * 4 + nnz_c * 4 + 4 * (m + 1)
+        numeric = nnz_a * (12 + vsize) + nprods * (4 + vsize) + nnz_c * (4 + 4 + vsize) + 4 * (m + 1)
+        return {"setup": setup, "symbolic": symbolic, "numeric": numeric}
     symbolic = nnz_a * 16 + nprods * (4 + 2) + 4 * (m + 1)
     numeric = nnz_a * (16 + vsize) + nprods * (4 + vsize + 2) + nnz_c * (4 + vsize) + 4 * (m + 1)
     return {"setup": setup, "symbolic": symbolic, "numeric": numeric}
@@ -472,6 +484,8 @@ def table_configs(msp, torch, dev, names, peak, flush):
         if "spgemm" in BJ_OPS[name]:
             reps = 3 if name == "C5" else 5
             rec = []
+            oc = ov = None  # C's arrays, preallocated after the first (untimed) call
+            path = None
             for i in range(reps + 2):
                 if small:
                     flush()
@@ -481,18 +495,22 @@ def table_configs(msp, torch, dev, names, peak, flush):
                 b = tm.ev()
                 p.symbolic()
                 c = tm.ev()
-                Cg = p.numeric()
+                Cg = p.numeric(col=oc, val=ov)
                 d = tm.ev()
                 if i >= 2:
                     rec.append((a, b, c, d))
                 nprods, nnzc = p.nprods, Cg.nnz
+                path = "row_accumulator" if p.info.row_accumulator > 0 else "esc_tiles"
+                if oc is None:
+                    oc, ov = Cg.col, Cg.val
                 del Cg, p
+            del oc, ov
             torch.cuda.synchronize(dev)
             ph = {k: float(np.mean([r[j].elapsed_time(r[j + 1]) for r in rec]))
                   for j, k in enumerate(("setup", "symbolic", "numeric"))}
             ms = sum(ph.values())
-            pb = spgemm_pass_bytes(A.m, A.nnz, nprods, nnzc, vs)
-            ent["spgemm"] = {"op": "A * A", "ms": ms, "nprods": nprods, "nnz_c": nnzc,
+            pb = spgemm_pass_bytes(A.m, A.nnz, nprods, nnzc, vs, path == "row_accumulator")
+            ent["spgemm"] = {"op": "A * A", "ms": ms, "nprods": nprods, "nnz_c": nnzc, "short_row_path": path,
                              "products_per_s": nprods / ms * 1e3,
                              "passes": {k: {"ms": ph[k], "alg_bytes": pb[k], "GB_s": pb[k] / ph[k] / 1e6,
                                             "frac_hbm": pb[k] / ph[k] / 1e6 / peak} for k in ph}}
@@ -639,6 +657,8 @@ def msp_arm(args):
     # events recorded on that same stream around each launch
     spmv_kernel_ms = []
 
+    gemm_out = [None, None]
+
     def step(timed: bool):
         e0 = tm.ev()
         if world > 1:
@@ -666,8 +686,10 @@ def msp_arm(args):
             P = msp.SpGemmPlan(A, Bg)
             P.setup()
             P.symbolic()
-            Cg = P.numeric()
+            Cg = P.numeric(col=gemm_out[0], val=gemm_out[1])
             g1 = tm.ev()
+            if gemm_out[0] is None:  # C's arrays kept for the following steps (warm-up allocates)
+                gemm_out[0], gemm_out[1] = Cg.col, Cg.val
             gm_ev = (g0, g1)
             extra["spgemm_nprods"] = P.nprods
             extra["spgemm_nnz_c"] = Cg.nnz
@@ -754,6 +776,7 @@ def msp_arm(args):
         def flush():
             flush_buf.fill_(1.0)
         A = At = y = Bfull = add_col = add_val = None  # noqa: F841  (free the headline workload's device memory)
+        gemm_out[0] = gemm_out[1] = None
         torch.cuda.empty_cache()
         table = table_configs(msp, torch, dev, [c for c in args.table_configs.split(",") if c], peak, flush)
         pred = predictability(table)

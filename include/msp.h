@@ -216,8 +216,10 @@ typedef struct {
                                 pass: output span <= 12288 columns and >= 1
                                 product per 4 columns of it (
                                 MSP_SPGEMM_SEGMENTED=0 disables) */
-    int64_t row_accumulator; /* 1: every short row's output span is at most
-                                65,536 columns, so the short rows take the
+    int64_t row_accumulator; /* > 0: every short row's output span is at most
+                                65,536 columns (the value is the widest
+                                span, which sizes the bitmaps), so the short
+                                rows take the
                                 row-accumulator path (a warp per row: bitmap
                                 count in symbolic, shared-memory accumulation
                                 in k order in numeric) and no product tile

@@ -293,8 +293,7 @@ spa_row_kernel(const int32_t *__restrict__ sparow, const int32_t *__restrict__ A
 // Every column sums its products in Gustavson's order with separate multiply
 // and add roundings, as the oracle does.  The choice is global (all short
 // rows or none) so that the tile pass is either skipped or untouched.
-constexpr int WR_SPAN = 65536;            // bitmap bits per warp (8 KB)
-constexpr int WR_WORDS = WR_SPAN / 32;
+constexpr int WR_SPAN = 65536;            // widest short-row span the bitmaps cover (8 KB per warp)
 constexpr int WR_SYM_WARPS = 8;           // 64 KB of bitmaps per CTA
 constexpr int WR_UMAX = 512;              // accumulator entries per warp per pass (6 KB with the column list)
 constexpr int WR_NUM_WARPS = 8;
@@ -315,7 +314,7 @@ __global__ void wr_span_kernel(int32_t m, const int32_t *__restrict__ Arp, const
 {
     const int lane = threadIdx.x & 31;
     const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
-    unsigned long long nfail = 0;
+    unsigned long long nfail = 0, mxspan = 0;
     for (int64_t r = int64_t(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5); r < m; r += nwarps) {
         if (rowlong[r]) continue;
         const int32_t a0 = Arp[r], a1 = Arp[r + 1];
@@ -332,15 +331,81 @@ __global__ void wr_span_kernel(int32_t m, const int32_t *__restrict__ Arp, const
         if (lane == 0) {
             lo_out[r] = lo;
             hi_out[r] = hi;
-            if (hi >= lo && int64_t(hi) - lo + 1 > WR_SPAN) ++nfail;
+            if (hi >= lo) {
+                const unsigned long long sp = (unsigned long long)(int64_t(hi) - lo + 1);
+                if (sp > WR_SPAN) ++nfail;
+                mxspan = sp > mxspan ? sp : mxspan;
+            }
         }
     }
     if (lane == 0 && nfail) atomicAdd(fail, nfail);
+    if (lane == 0 && mxspan) atomicMax(fail + 1, mxspan);
 }
 
-// Symbolic: bitmap mark, count, ascending column list at ucol + S[rp[r]].
-__global__ void __launch_bounds__(WR_SYM_WARPS * 32)
-wr_symbolic_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
+// One step per A nonzero of a chunk of <= 32 (lane l holds nonzero l's B
+// row start b0 and length): f(step, c[u], v[u]) for 8 steps at a time, the
+// 8 steps' B entries loaded up front (lane q holds entry q of the step's B
+// row; rows longer than a warp take the per-step loop).  f runs in step
+// order; `sync` adds a __syncwarp after every step (numeric ordering).
+template <bool VALS, typename V, class F>
+__device__ __forceinline__ void wr_steps(int nl, int lane, int32_t b0, int32_t len, const int32_t *__restrict__ Bcol,
+                                         const V *__restrict__ Bval, bool sync, F &&f)
+{
+    if (__all_sync(0xffffffffu, len <= 32)) {
+        for (int s0 = 0; s0 < nl; s0 += 8) {
+            int32_t c[8];
+            V v[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+                const int sidx = (s0 + u) & 31;
+                const int32_t bb = __shfl_sync(0xffffffffu, b0, sidx);
+                const int32_t ll = __shfl_sync(0xffffffffu, len, sidx);
+                const bool ok = s0 + u < nl && lane < ll;
+                c[u] = ok ? Bcol[bb + lane] : -1;
+                if constexpr (VALS) v[u] = ok ? Bval[bb + lane] : V(0);
+            }
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+                f(s0 + u, c[u], VALS ? v[u] : V(0));
+                if (sync) __syncwarp();
+            }
+        }
+    } else {
+        for (int sidx = 0; sidx < nl; ++sidx) {
+            const int32_t bb = __shfl_sync(0xffffffffu, b0, sidx);
+            const int32_t ll = __shfl_sync(0xffffffffu, len, sidx);
+            for (int q0 = 0; q0 < ll; q0 += 32) {
+                const bool ok = q0 + lane < ll;
+                const int32_t c = ok ? Bcol[bb + q0 + lane] : -1;
+                V v = V(0);
+                if constexpr (VALS) v = ok ? Bval[bb + q0 + lane] : V(0);
+                f(sidx, c, v);
+            }
+            if (sync) __syncwarp();
+        }
+    }
+}
+
+// Position of the n-th (0-based) set bit of w (w has more than n set bits).
+__device__ __forceinline__ int nth_set_bit(uint32_t w, int n)
+{
+    int pos = 0;
+#pragma unroll
+    for (int sh = 16; sh >= 1; sh >>= 1) {
+        const int c = __popc(w & ((1u << sh) - 1u));
+        if (n >= c) {
+            n -= c;
+            w >>= sh;
+            pos += sh;
+        }
+    }
+    return pos;
+}
+
+// Symbolic: bitmap mark, then ONE pass over the bitmap (4 words per lane per
+// round) counts the columns and writes them ascending at ucol + S[rp[r]].
+__global__ void __launch_bounds__(WR_SYM_WARPS * 32, 1)
+wr_symbolic_kernel(int32_t m, int nw_max, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
                    const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
                    const uint8_t *__restrict__ rowlong, const int64_t *__restrict__ S,
                    const int32_t *__restrict__ spanlo, const int32_t *__restrict__ spanhi,
@@ -348,7 +413,7 @@ wr_symbolic_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__
 {
     extern __shared__ __align__(16) uint32_t wr_bm_all[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    uint32_t *bm = wr_bm_all + warp * WR_WORDS;
+    uint32_t *bm = wr_bm_all + size_t(warp) * nw_max;  // nw_max: a multiple of 128 words
     const int64_t nwarps = int64_t(gridDim.x) * WR_SYM_WARPS;
     for (int64_t r = int64_t(blockIdx.x) * WR_SYM_WARPS + warp; r < m; r += nwarps) {
         if (rowlong[r]) continue;
@@ -358,166 +423,199 @@ wr_symbolic_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__
             continue;
         }
         const int nw = (hi - lo + 32) >> 5;
-        for (int w = lane; w < nw; w += 32) bm[w] = 0u;
+        const int nq = (nw + 127) >> 7;  // rounds of 4 words per lane
+        for (int q = 0; q < nq; ++q) reinterpret_cast<uint4 *>(bm)[q * 32 + lane] = make_uint4(0u, 0u, 0u, 0u);
         __syncwarp();
         const int32_t a0 = Arp[r], a1 = Arp[r + 1];
         for (int32_t jc = a0; jc < a1; jc += 32) {
             const int32_t j = jc + lane;
-            const int nl = min(32, a1 - jc);
             int32_t b0 = 0, len = 0;
             if (j < a1) {
                 const int32_t k = Acol[j];
                 b0 = Brp[k];
                 len = Brp[k + 1] - b0;
             }
-            int tot;
-            const int off = warp_excl_sum(len, lane, &tot);
-            // products of the chunk, flattened over the lanes, 8 loads in flight per lane
-            for (int t0 = 0; t0 < tot; t0 += 32 * 8) {
-                int32_t c[8];
-#pragma unroll
-                for (int u = 0; u < 8; ++u) {
-                    const int t = t0 + u * 32 + lane;
-                    int sidx = 0;  // lane owning product t: the last lane with off <= t
-#pragma unroll
-                    for (int step = 16; step >= 1; step >>= 1) {
-                        const int cand = sidx + step;
-                        const int oc = __shfl_sync(0xffffffffu, off, cand & 31);
-                        if (cand < nl && oc <= t) sidx = cand;
-                    }
-                    const int ob = __shfl_sync(0xffffffffu, off, sidx);
-                    const int32_t bb = __shfl_sync(0xffffffffu, b0, sidx);
-                    c[u] = t < tot ? Bcol[bb + (t - ob)] : -1;
+            wr_steps<false, float>(min(32, a1 - jc), lane, b0, len, Bcol, nullptr, false, [&](int, int32_t c, float) {
+                if (c >= 0) {
+                    const int x = c - lo;
+                    atomicOr(&bm[x >> 5], 1u << (x & 31));
                 }
-#pragma unroll
-                for (int u = 0; u < 8; ++u)
-                    if (c[u] >= 0) {
-                        const int x = c[u] - lo;
-                        atomicOr(&bm[x >> 5], 1u << (x & 31));
-                    }
-            }
+            });
         }
         __syncwarp();
-        int cnt = 0;
-        for (int w = lane; w < nw; w += 32) cnt += __popc(bm[w]);
-        cnt = __reduce_add_sync(0xffffffffu, cnt);
-        if (lane == 0) Crp_counts[r] = cnt;
-        // ascending column list at the row's product offset
         int32_t *dst = ucol + S[a0];
         int run = 0;
-        for (int w0 = 0; w0 < nw; w0 += 32) {
-            const int w = w0 + lane;
-            uint32_t word = w < nw ? bm[w] : 0u;
-            int wt;
-            int p = run + warp_excl_sum(__popc(word), lane, &wt);
-            while (word) {
-                const int b = __ffs(word) - 1;
-                word &= word - 1;
-                dst[p++] = lo + w * 32 + b;
+        for (int q = 0; q < nq; ++q) {
+            const uint4 w4 = reinterpret_cast<const uint4 *>(bm)[q * 32 + lane];
+            const int p0 = __popc(w4.x), p1 = __popc(w4.y), p2 = __popc(w4.z), p3 = __popc(w4.w);
+            int tot;
+            const int ex = warp_excl_sum(p0 + p1 + p2 + p3, lane, &tot);
+            // the round's tot columns go out converged and coalesced: output o
+            // (o = lane, lane + 32, ...) finds the lane owning it (last lane
+            // with ex <= o), the word within that lane's four, and the bit
+            for (int o0 = 0; o0 < tot; o0 += 32) {
+                const int o = o0 + lane;
+                int src_l = 0;
+#pragma unroll
+                for (int step = 16; step >= 1; step >>= 1) {
+                    const int cand = src_l + step;
+                    if (__shfl_sync(0xffffffffu, ex, cand) <= o) src_l = cand;
+                }
+                const int rel = o - __shfl_sync(0xffffffffu, ex, src_l);
+                const uint32_t x0 = __shfl_sync(0xffffffffu, w4.x, src_l), x1 = __shfl_sync(0xffffffffu, w4.y, src_l);
+                const uint32_t x2 = __shfl_sync(0xffffffffu, w4.z, src_l), x3 = __shfl_sync(0xffffffffu, w4.w, src_l);
+                const int c0 = __popc(x0), c1 = c0 + __popc(x1), c2 = c1 + __popc(x2);
+                int e, nth;
+                uint32_t word;
+                if (rel < c0) { e = 0; nth = rel; word = x0; }
+                else if (rel < c1) { e = 1; nth = rel - c0; word = x1; }
+                else if (rel < c2) { e = 2; nth = rel - c1; word = x2; }
+                else { e = 3; nth = rel - c2; word = x3; }
+                const int b = nth_set_bit(word, nth);
+                if (o < tot) dst[run + o] = lo + (q * 128 + src_l * 4 + e) * 32 + b;
             }
-            run += wt;
+            run += tot;
         }
+        if (lane == 0) Crp_counts[r] = run;
         __syncwarp();  // the bitmap is reused by the warp's next row
     }
 }
 
-// Numeric: accumulate into shared memory in k order, WR_UMAX columns per pass.
+// Numeric: a hash of the row's column list (16-bit column offset | 16-bit
+// rank per 32-bit slot, linear probing) gives each product's rank in one or
+// two shared-memory probes; products accumulate into shared memory in k
+// order.  WR_UMAX columns per pass.
+constexpr int WR_HSLOTS = 2 * WR_UMAX;
+constexpr uint32_t WR_EMPTY = 0xffffffffu;
+constexpr int WR_NUM_SMEM = WR_NUM_WARPS * (WR_UMAX * 8 + WR_HSLOTS * 4);
+
+__device__ __forceinline__ uint32_t wr_hash(uint32_t x) { return (x * 0x9E3779B1u) >> (32 - 10); }
+static_assert(WR_HSLOTS == 1024, "wr_hash yields 10 bits");
+
 template <typename V>
-__global__ void __launch_bounds__(WR_NUM_WARPS * 32)
+__global__ void __launch_bounds__(WR_NUM_WARPS * 32, 3)
 wr_numeric_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
                   const V *__restrict__ Aval, const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
                   const V *__restrict__ Bval, const uint8_t *__restrict__ rowlong, const int64_t *__restrict__ S,
-                  const int32_t *__restrict__ ucol, const int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol,
-                  V *__restrict__ Cval)
+                  const int32_t *__restrict__ spanlo, const int32_t *__restrict__ ucol,
+                  const int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol, V *__restrict__ Cval)
 {
-    __shared__ int32_t s_uc[WR_NUM_WARPS][WR_UMAX];
-    __shared__ double s_acc[WR_NUM_WARPS][WR_UMAX];
+    extern __shared__ __align__(16) char wr_num_smem[];  // [warps][WR_UMAX] acc, then [warps][WR_HSLOTS] hash
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    int32_t *uc = s_uc[warp];
-    double *acc = s_acc[warp];
+    double *acc = reinterpret_cast<double *>(wr_num_smem) + warp * WR_UMAX;
+    uint32_t *tab = reinterpret_cast<uint32_t *>(wr_num_smem + WR_NUM_WARPS * WR_UMAX * 8) + warp * WR_HSLOTS;
     const int64_t nwarps = int64_t(gridDim.x) * WR_NUM_WARPS;
-    for (int64_t r = int64_t(blockIdx.x) * WR_NUM_WARPS + warp; r < m; r += nwarps) {
-        if (rowlong[r]) continue;
-        const int32_t cb = Crp[r], U = Crp[r + 1] - cb;
-        if (U == 0) continue;
-        const int32_t a0 = Arp[r], a1 = Arp[r + 1];
-        const int32_t *src = ucol + S[a0];
+    // The next row's header, its list offset and the first 4 x 32 entries of
+    // its column list are loaded while the current row accumulates (rows of
+    // one warp are independent), hiding their latency chain.
+    struct Hdr {
+        int32_t cb, ce, a0, a1, lo, skip;
+    };
+    auto load_hdr = [&](int64_t rr) {
+        Hdr h{0, 0, 0, 0, 0, 1};
+        if (rr < m) {
+            h.skip = rowlong[rr];
+            h.cb = Crp[rr];
+            h.ce = Crp[rr + 1];
+            h.a0 = Arp[rr];
+            h.a1 = Arp[rr + 1];
+            h.lo = spanlo[rr];
+        }
+        return h;
+    };
+    int64_t r = int64_t(blockIdx.x) * WR_NUM_WARPS + warp;
+    Hdr cur = load_hdr(r);
+    int64_t cur_off = (cur.skip || cur.ce == cur.cb) ? 0 : S[cur.a0];
+    int32_t pre[4];  // entries lane + 32 u of the current row's column list
+#pragma unroll
+    for (int u = 0; u < 4; ++u) pre[u] = (lane + 32 * u < cur.ce - cur.cb) ? ucol[cur_off + lane + 32 * u] : 0;
+    for (; r < m; r += nwarps) {
+        const Hdr nxt = load_hdr(r + nwarps);
+        const int32_t cb = cur.cb, U = cur.ce - cur.cb;
+        const bool work = !cur.skip && U > 0;
+        if (work) {
+        const int32_t a0 = cur.a0, a1 = cur.a1;
+        const int32_t lo = cur.lo;
+        const int32_t *src = ucol + cur_off;
+        // the first chunk of A nonzeros is loaded before the hash build, so
+        // its dependent B-row offsets are in flight meanwhile (reused by
+        // every column pass)
+        int32_t f_b0 = 0, f_len = 0;
+        double f_av = 0.0;
+        {
+            const int32_t j = a0 + lane;
+            if (j < a1) {
+                const int32_t k = Acol[j];
+                f_av = double(Aval[j]);
+                f_b0 = Brp[k];
+                f_len = Brp[k + 1] - f_b0;
+            }
+        }
         for (int cs = 0; cs < U; cs += WR_UMAX) {
             const int nu = min(WR_UMAX, U - cs);
-            for (int i = lane; i < nu; i += 32) {
-                uc[i] = src[cs + i];
-                acc[i] = -0.0;  // -0 + p == p for every p: the first product needs no special case
-            }
+            for (int i = lane; i < WR_HSLOTS; i += 32) tab[i] = WR_EMPTY;
+            for (int i = lane; i < nu; i += 32) acc[i] = -0.0;  // -0 + p == p for every p
             __syncwarp();
-            const int32_t cmin = uc[0], cmax = uc[nu - 1];
+            auto insert = [&](int i, int32_t col) {
+                const uint32_t x = uint32_t(col - lo);
+                uint32_t h = wr_hash(x);
+                while (atomicCAS(&tab[h], WR_EMPTY, x | (uint32_t(i) << 16)) != WR_EMPTY) h = (h + 1) & (WR_HSLOTS - 1);
+            };
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                const int i = lane + 32 * t;
+                if (i < nu) insert(i, cs == 0 ? pre[t] : src[cs + i]);
+            }
+            for (int i = lane + 128; i < nu; i += 32) insert(i, src[cs + i]);
+            __syncwarp();
+            const int32_t cmin = src[cs], cmax = src[cs + nu - 1];
             for (int32_t jc = a0; jc < a1; jc += 32) {
                 const int32_t j = jc + lane;
-                const int nl = min(32, a1 - jc);
-                int32_t b0 = 0, len = 0;
-                double av = 0.0;
-                if (j < a1) {
-                    const int32_t k = Acol[j];
-                    b0 = Brp[k];
-                    len = Brp[k + 1] - b0;
-                    av = double(Aval[j]);
-                }
-                if (__all_sync(0xffffffffu, len <= 32)) {
-                    // one B row per step, lane q holds its q-th entry; 8 steps of loads in flight
-                    for (int s0 = 0; s0 < nl; s0 += 8) {
-                        int32_t c[8];
-                        V v[8];
-#pragma unroll
-                        for (int u = 0; u < 8; ++u) {
-                            const int sidx = s0 + u;
-                            const int32_t bb = __shfl_sync(0xffffffffu, b0, sidx & 31);
-                            const int32_t ll = __shfl_sync(0xffffffffu, len, sidx & 31);
-                            const bool ok = sidx < nl && lane < ll;
-                            c[u] = ok ? Bcol[bb + lane] : -1;
-                            v[u] = ok ? Bval[bb + lane] : V(0);
-                        }
-#pragma unroll
-                        for (int u = 0; u < 8; ++u) {
-                            const double a = __shfl_sync(0xffffffffu, av, (s0 + u) & 31);
-                            if (c[u] >= cmin && c[u] <= cmax) {
-                                int lo = 0, hi = nu - 1;  // rank of c in the column list
-                                while (lo < hi) {
-                                    const int mid = (lo + hi) >> 1;
-                                    if (uc[mid] < c[u]) lo = mid + 1;
-                                    else hi = mid;
-                                }
-                                acc[lo] = __dadd_rn(acc[lo], __dmul_rn(a, double(v[u])));
-                            }
-                            __syncwarp();  // the next k's sums follow this one's
-                        }
-                    }
-                } else {
-                    for (int sidx = 0; sidx < nl; ++sidx) {
-                        const int32_t bb = __shfl_sync(0xffffffffu, b0, sidx);
-                        const int32_t ll = __shfl_sync(0xffffffffu, len, sidx);
-                        const double a = __shfl_sync(0xffffffffu, av, sidx);
-                        for (int q = lane; q < ll; q += 32) {
-                            const int32_t c = Bcol[bb + q];
-                            if (c >= cmin && c <= cmax) {
-                                int lo = 0, hi = nu - 1;
-                                while (lo < hi) {
-                                    const int mid = (lo + hi) >> 1;
-                                    if (uc[mid] < c) lo = mid + 1;
-                                    else hi = mid;
-                                }
-                                acc[lo] = __dadd_rn(acc[lo], __dmul_rn(a, double(Bval[bb + q])));
-                            }
-                        }
-                        __syncwarp();
+                int32_t b0 = f_b0, len = f_len;
+                double av = f_av;
+                if (jc != a0) {
+                    b0 = 0;
+                    len = 0;
+                    av = 0.0;
+                    if (j < a1) {
+                        const int32_t k = Acol[j];
+                        b0 = Brp[k];
+                        len = Brp[k + 1] - b0;
+                        av = double(Aval[j]);
                     }
                 }
+                wr_steps<true, V>(min(32, a1 - jc), lane, b0, len, Bcol, Bval, true, [&](int sidx, int32_t c, V v) {
+                    const double a = __shfl_sync(0xffffffffu, av, sidx & 31);
+                    if (c >= cmin && c <= cmax) {
+                        const uint32_t x = uint32_t(c - lo);
+                        uint32_t h = wr_hash(x), e;
+                        while (((e = tab[h]) & 0xffffu) != x || e == WR_EMPTY) h = (h + 1) & (WR_HSLOTS - 1);
+                        const int rk = int(e >> 16);
+                        acc[rk] = __dadd_rn(acc[rk], __dmul_rn(a, double(v)));
+                    }
+                });
             }
             __syncwarp();
-            for (int i = lane; i < nu; i += 32) {
-                Ccol[cb + cs + i] = uc[i];
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                const int i = lane + 32 * t;
+                if (i < nu) {
+                    Ccol[cb + cs + i] = cs == 0 ? pre[t] : src[cs + i];
+                    Cval[cb + cs + i] = V(acc[i]);
+                }
+            }
+            for (int i = lane + 128; i < nu; i += 32) {
+                Ccol[cb + cs + i] = src[cs + i];
                 Cval[cb + cs + i] = V(acc[i]);
             }
             __syncwarp();
         }
+        }
+        // the next row's list offset and first entries
+        cur = nxt;
+        cur_off = (cur.skip || cur.ce == cur.cb) ? 0 : S[cur.a0];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) pre[u] = (lane + 32 * u < cur.ce - cur.cb) ? ucol[cur_off + lane + 32 * u] : 0;
     }
 }
 
@@ -532,7 +630,8 @@ struct SetupWs {
     int64_t *longO;      // [m + 1] prefix of longP
     int64_t *longC;      // [m]  chunks of the i-th long row
     int64_t *longCO;     // [m + 1] prefix of longC
-    unsigned long long *stats;  // [8]: [0] max row products, [1..6] gathered setup sizes
+    unsigned long long *stats;  // [16]: [0] max row products, [1..6] gathered setup sizes, [7] short rows
+                                //       too wide for the row accumulator, [8] widest short-row span
     int32_t *spanlo, *spanhi;   // [m] output column span of each long row (segmented path, f3)
     int32_t *spaflag;           // [m] 1 = the row takes the segmented path
     int64_t *spapos;            // [m + 1]
@@ -557,7 +656,7 @@ SetupWs carve_setup(const msp_csr *A, void *ws, size_t cap, bool *ok)
     w.longO = cv.take<int64_t>(size_t(m + 1));
     w.longC = cv.take<int64_t>(size_t(m > 0 ? m : 1));
     w.longCO = cv.take<int64_t>(size_t(m + 1));
-    w.stats = cv.take<unsigned long long>(8);
+    w.stats = cv.take<unsigned long long>(16);
     w.spanlo = cv.take<int32_t>(size_t(m > 0 ? m : 1));
     w.spanhi = cv.take<int32_t>(size_t(m > 0 ? m : 1));
     w.spaflag = cv.take<int32_t>(size_t(m > 0 ? m : 1));
@@ -1232,7 +1331,8 @@ __global__ void info_gather_kernel(const int64_t *__restrict__ S, int64_t nnzA, 
     out[3] = nlong > 0 ? longCO[nlong] : 0;
     out[4] = int64_t(stats[0]);
     out[5] = spapos[m];
-    // out[6] is stats[7] itself: short rows whose span is too wide for the row accumulator
+    // out[6], out[7] are stats[7], stats[8] themselves: short rows too wide for
+    // the row accumulator, widest short-row span
 }
 
 // A pinned host staging word array per host thread for the synchronising reads.
@@ -1261,8 +1361,8 @@ msp_status read_info(const SetupWs &sw, int64_t m, int64_t nnzA, HostInfo *h, cu
                                         reinterpret_cast<int64_t *>(sw.stats) + 1);
     msp_status st = last_launch("info_gather_kernel");
     if (st != MSP_OK) return st;
-    int64_t v[7];
-    st = read_back(reinterpret_cast<const int64_t *>(sw.stats) + 1, 7, v, s, "spgemm: setup sizes");
+    int64_t v[8];
+    st = read_back(reinterpret_cast<const int64_t *>(sw.stats) + 1, 8, v, s, "spgemm: setup sizes");
     if (st != MSP_OK) return st;
     h->nprods = v[0];
     h->nlong = v[1];
@@ -1270,7 +1370,8 @@ msp_status read_info(const SetupWs &sw, int64_t m, int64_t nnzA, HostInfo *h, cu
     h->LC = v[3];
     h->maxP = v[4];
     h->nspa = v[5];
-    h->rowacc = (rowacc_enabled() && v[6] == 0) ? 1 : 0;
+    // row accumulator: 0 = off, else the widest short-row span (sizes the bitmaps)
+    h->rowacc = (rowacc_enabled() && v[6] == 0) ? std::max<int64_t>(v[7], 1) : 0;
     return MSP_OK;
 }
 
@@ -1356,42 +1457,53 @@ bool rowacc_enabled()
 }
 
 template <bool NUM>
-msp_status run_rowacc(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, int32_t *Crp,
-                      int32_t *Ccol, void *Cval, cudaStream_t s)
+msp_status run_rowacc(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, int64_t rowacc_span,
+                      int32_t *Crp, int32_t *Ccol, void *Cval, cudaStream_t s)
 {
     const int32_t m = A->nrows;
     if (!NUM) {
-        const int smem = WR_SYM_WARPS * WR_WORDS * 4;
-        int occ = 1;
-        msp_status st = set_smem_attr(reinterpret_cast<const void *>(wr_symbolic_kernel), smem,
-                                      "spgemm: row accumulator smem", WR_SYM_WARPS * 32, &occ, true);
+        // bitmap words per warp: the widest short row's span, in rounds of 128 words
+        const int nw_max = int(ceil_div(ceil_div(rowacc_span, 32), 128) * 128);
+        const int smem = WR_SYM_WARPS * nw_max * 4;
+        // the carveout / occupancy query is per bitmap size: no per-kernel cache here
+        msp_status st = cuda_check(cudaFuncSetAttribute(reinterpret_cast<const void *>(wr_symbolic_kernel),
+                                                        cudaFuncAttributeMaxDynamicSharedMemorySize, smem),
+                                   "spgemm: row accumulator smem");
         if (st != MSP_OK) return st;
+        int occ = 1;
+        st = cuda_check(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, wr_symbolic_kernel, WR_SYM_WARPS * 32,
+                                                                      size_t(smem)),
+                        "spgemm: row accumulator occupancy");
+        if (st != MSP_OK) return st;
+        if (occ < 1) occ = 1;
         const int64_t g = std::min<int64_t>(int64_t(occ) * sm_count(), ceil_div(m, WR_SYM_WARPS));
         wr_symbolic_kernel<<<unsigned(g > 0 ? g : 1), WR_SYM_WARPS * 32, smem, s>>>(
-            m, A->row_offsets, A->col_idx, B->row_offsets, B->col_idx, sw.rowlong, sw.S, sw.spanlo, sw.spanhi,
-            Crp + 1, mw.ucol);
+            m, nw_max, A->row_offsets, A->col_idx, B->row_offsets, B->col_idx, sw.rowlong, sw.S, sw.spanlo,
+            sw.spanhi, Crp + 1, mw.ucol);
         return last_launch("wr_symbolic_kernel");
     }
     if (A->dtype == MSP_F64) {
         auto kern = wr_numeric_kernel<double>;
         int occ = 1;
-        msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), 0, "spgemm: row accumulator",
+        msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), WR_NUM_SMEM, "spgemm: row accumulator",
                                       WR_NUM_WARPS * 32, &occ, true);
         if (st != MSP_OK) return st;
         const int64_t g = std::min<int64_t>(int64_t(occ) * sm_count(), ceil_div(m, WR_NUM_WARPS));
-        kern<<<unsigned(g > 0 ? g : 1), WR_NUM_WARPS * 32, 0, s>>>(
+        kern<<<unsigned(g > 0 ? g : 1), WR_NUM_WARPS * 32, WR_NUM_SMEM, s>>>(
             m, A->row_offsets, A->col_idx, static_cast<const double *>(A->vals), B->row_offsets, B->col_idx,
-            static_cast<const double *>(B->vals), sw.rowlong, sw.S, mw.ucol, Crp, Ccol, static_cast<double *>(Cval));
+            static_cast<const double *>(B->vals), sw.rowlong, sw.S, sw.spanlo, mw.ucol, Crp, Ccol,
+            static_cast<double *>(Cval));
     } else {
         auto kern = wr_numeric_kernel<float>;
         int occ = 1;
-        msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), 0, "spgemm: row accumulator",
+        msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), WR_NUM_SMEM, "spgemm: row accumulator",
                                       WR_NUM_WARPS * 32, &occ, true);
         if (st != MSP_OK) return st;
         const int64_t g = std::min<int64_t>(int64_t(occ) * sm_count(), ceil_div(m, WR_NUM_WARPS));
-        kern<<<unsigned(g > 0 ? g : 1), WR_NUM_WARPS * 32, 0, s>>>(
+        kern<<<unsigned(g > 0 ? g : 1), WR_NUM_WARPS * 32, WR_NUM_SMEM, s>>>(
             m, A->row_offsets, A->col_idx, static_cast<const float *>(A->vals), B->row_offsets, B->col_idx,
-            static_cast<const float *>(B->vals), sw.rowlong, sw.S, mw.ucol, Crp, Ccol, static_cast<float *>(Cval));
+            static_cast<const float *>(B->vals), sw.rowlong, sw.S, sw.spanlo, mw.ucol, Crp, Ccol,
+            static_cast<float *>(Cval));
     }
     return last_launch("wr_numeric_kernel");
 }
@@ -1479,7 +1591,7 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
     SetupWs w = carve_setup(A, ws1, b1, &ok);
     if (!ok) return MSP_ERR_WORKSPACE;
     const int64_t m = A->nrows, nnz = A->nnz;
-    msp_status st = cuda_check(cudaMemsetAsync(w.stats, 0, 8 * sizeof(unsigned long long), s), "spgemm: clear");
+    msp_status st = cuda_check(cudaMemsetAsync(w.stats, 0, 16 * sizeof(unsigned long long), s), "spgemm: clear");
     if (st != MSP_OK) return st;
     if (nnz > 0) {
         const int64_t thr = ceil_div(m + nnz, AROW_ITEMS);
@@ -1508,7 +1620,7 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
         if (nnz > 0 && rowacc_enabled()) {  // short-row spans for the row accumulator
             wr_span_kernel<<<unsigned(std::min<int64_t>(ceil_div(m, 8), 148 * 16)), 256, 0, s>>>(
                 A->nrows, A->row_offsets, A->col_idx, B->row_offsets, B->col_idx, w.rowlong, w.spanlo, w.spanhi,
-                &w.stats[7]);
+                &w.stats[7]);  // [7] too-wide rows, [8] widest span
             st = last_launch("wr_span_kernel");
             if (st != MSP_OK) return st;
         }
@@ -1607,7 +1719,7 @@ msp_status spgemm_pass(const msp_csr *A, const msp_csr *B, const void *ws1, size
         return MSP_ERR_ARG;
     }
     if (h.nprods > 0 && m > 0) {
-        if (h.rowacc) st = run_rowacc<NUM>(A, B, sw, mw, Crp, Ccol, Cval, s);
+        if (h.rowacc) st = run_rowacc<NUM>(A, B, sw, mw, h.rowacc, Crp, Ccol, Cval, s);
         else
             st = (A->dtype == MSP_F64) ? run_tiles<double, NUM>(A, B, sw, mw, ntiles, maxspan, Crp, Ccol, Cval, s)
                                        : run_tiles<float, NUM>(A, B, sw, mw, ntiles, maxspan, Crp, Ccol, Cval, s);

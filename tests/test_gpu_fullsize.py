@@ -53,7 +53,7 @@ def test_c2_spgemm_full_complete():
     A = gen.config("C2", "random")
     info = assert_spgemm_complete(A, A, "C2 A*A")
     assert info.nprods == 890 ** 3
-    assert info.row_accumulator == 1  # stencil rows: the short-row accumulator path
+    assert info.row_accumulator == 2 * (2 + 2 * 100 + 2 * 100 ** 2) + 1  # stencil rows: accumulator path, widest span
 
 
 def test_c4_spgemm_full_complete():

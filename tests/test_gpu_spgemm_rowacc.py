@@ -53,12 +53,12 @@ def test_taken_on_stencils():
     for name in ("C1",):
         A = gen.config(name, "int")
         info = check(A, A, name, exact=True)
-        assert info.row_accumulator == 1 and info.ntiles == 0
+        assert info.row_accumulator > 0 and info.ntiles == 0
     A = gen.config("C2", "random")
     p_rows = slice(0, 20001)
     S = gen.CSR(20000, A.n, A.rp[p_rows] - A.rp[0], A.col[:A.rp[20000]], A.val[:A.rp[20000]])
     info = check(S, A, "C2 rows [0, 20000) x A")
-    assert info.row_accumulator == 1
+    assert info.row_accumulator > 0
 
 
 def test_many_unique_columns_and_long_b_rows():
@@ -74,7 +74,7 @@ def test_many_unique_columns_and_long_b_rows():
     Arp, Acol = _rows(alens, k, rng)
     A = gen.CSR(400, k, Arp, Acol, gen.matrices.random_values(Acol.size, 3))
     info = check(A, B, "wide rows")
-    assert info.row_accumulator == 1
+    assert info.row_accumulator > 0
     W, _, _ = oracle.spgemm(A, B)
     assert np.diff(W.rp).max() > 512, "no row needs a second accumulator pass"
     Ai = A.with_values(gen.int_values(A.nnz, 4))
@@ -93,7 +93,7 @@ def test_signed_zero_and_cancellation():
                 np.array([3.0, 5.0, 3.0, -0.0]))
     rp, col, val, info = run(A, B)
     W, _, _ = oracle.spgemm(A, B)
-    assert info.row_accumulator == 1
+    assert info.row_accumulator > 0
     assert np.array_equal(rp, W.rp) and np.array_equal(col, W.col)
     assert np.array_equal(val.view(np.uint64), W.val.view(np.uint64)), (val, W.val)
 
