@@ -132,10 +132,17 @@ def spadd_alg_bytes(m, nnz_a, nnz_b, nnz_c, vsize):
     return (nnz_a + nnz_b) * (4 + vsize) + nnz_c * (4 + vsize) + 3 * 4 * (m + 1)
 
 
-def spgemm_pass_bytes(m, nnz_a, nprods, nnz_c, vsize, rowacc=False):
-    """The method's own traffic per pass.  Row accumulator
-    (rowacc): setup as below plus the span pass (A columns, 8 of B offsets
-    and 8 of B columns per A nonzero); symbolic reads A columns and B offsets
+def spgemm_pass_bytes(m, nnz_a, nprods, nnz_c, vsize, rowacc=False, small=False):
+    """The method's own traffic per pass.  Small-row path
+    (small, every short row has few products): setup as below plus the B row
+    start of every A nonzero (4) and the row classification (A offsets and 16
+    of S per row); symbolic reads each A nonzero's B row start and S (12),
+    gathers one B column per product (4), reads A offsets and S per row (24)
+    and writes C's row counts (4 per row); numeric reads the same plus A
+    values (12 + s per A nonzero), C's row offsets (8 per row), gathers a B
+    column + value per product (4 + s) and writes C (4 + s per C nonzero).
+    Row accumulator (rowacc): setup as below plus the span pass (A columns,
+    8 of B offsets and 8 of B columns per A nonzero); symbolic reads A columns and B offsets
     (12 per A nonzero), gathers one B column per product (4) and writes each
     row's column list (4 per C nonzero); numeric reads the same plus A values
     (12 + s per A nonzero), gathers a B column + value per product (4 + s),
@@ -150,6 +157,11 @@ def spgemm_pass_bytes(m, nnz_a, nprods, nnz_c, vsize, rowacc=False):
                 one B column + value gathered per product (4 + s), the
                 permutation read (2), C columns + values written (4 + s)."""
     setup = 4 * (m + 1) + nnz_a * (4 + 8 + 8 + 4)
+    if small:
+        setup += nnz_a * 4 + m * (8 + 16)
+        symbolic = nnz_a * 12 + nprods * 4 + m * (24 + 4)
+        numeric = nnz_a * (12 + vsize) + nprods * (4 + vsize) + nnz_c * (4 + vsize) + m * (24 + 8)
+        return {"setup": setup, "symbolic": symbolic, "numeric": numeric}
     if rowacc:
         setup += 4 * (m + 1) + nnz_a * (4 + 8 + 8)
         symbolic = nnz_a * 12 + nprods * 4 + nnz_c * 4 + 4 * (m + 1)
@@ -500,7 +512,12 @@ def table_configs(msp, torch, dev, names, peak, flush):
                 if i >= 2:
                     rec.append((a, b, c, d))
                 nprods, nnzc = p.nprods, Cg.nnz
-                path = "row_accumulator" if p.info.row_accumulator > 0 else "esc_tiles"
+                inf = p.info
+                path = ("esc_tiles" if inf.row_accumulator == 0 else
+                        "small_rows" if inf.bitmap_rows == 0 else
+                        "row_accumulator" if inf.small_rows == 0 else "small_rows+row_accumulator")
+                rows_by_path = {"small": int(inf.small_rows), "bitmap": int(inf.bitmap_rows),
+                                "long": int(inf.long_rows), "segmented": int(inf.segmented_rows)}
                 if oc is None:
                     oc, ov = Cg.col, Cg.val
                 del Cg, p
@@ -509,8 +526,9 @@ def table_configs(msp, torch, dev, names, peak, flush):
             ph = {k: float(np.mean([r[j].elapsed_time(r[j + 1]) for r in rec]))
                   for j, k in enumerate(("setup", "symbolic", "numeric"))}
             ms = sum(ph.values())
-            pb = spgemm_pass_bytes(A.m, A.nnz, nprods, nnzc, vs, path == "row_accumulator")
+            pb = spgemm_pass_bytes(A.m, A.nnz, nprods, nnzc, vs, path == "row_accumulator", path == "small_rows")
             ent["spgemm"] = {"op": "A * A", "ms": ms, "nprods": nprods, "nnz_c": nnzc, "short_row_path": path,
+                             "rows_by_path": rows_by_path,
                              "products_per_s": nprods / ms * 1e3,
                              "passes": {k: {"ms": ph[k], "alg_bytes": pb[k], "GB_s": pb[k] / ph[k] / 1e6,
                                             "frac_hbm": pb[k] / ph[k] / 1e6 / peak} for k in ph}}

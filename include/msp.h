@@ -64,7 +64,7 @@
 extern "C" {
 #endif
 
-#define MSP_VERSION 5  /* 2: msp_spgemm_info passed to symbolic / numeric; 3: segmented_rows; 4: msp_set_operation_async, msp_spadd_fused; 5: row_accumulator */
+#define MSP_VERSION 6  /* 2: msp_spgemm_info passed to symbolic / numeric; 3: segmented_rows; 4: msp_set_operation_async, msp_spadd_fused; 5: row_accumulator; 6: small_rows, bitmap_rows */
 
 typedef enum {
     MSP_OK = 0,
@@ -227,6 +227,18 @@ typedef struct {
                                 one int32 per product (each short row's column
                                 list) instead of the tile permutations.
                                 MSP_SPGEMM_ROWACC=0 disables (ablation). */
+    int64_t small_rows;      /* short rows with at most 64 products taking the
+                                compare-count path (a warp per batch of
+                                consecutive rows with <= 256 products: each
+                                product's rank from the first occurrences of
+                                its row, k-ordered sums; no column list in
+                                main_ws).  Short rows with more products whose
+                                span exceeds 65,536 columns are promoted to
+                                long rows, so the warp-row path covers every
+                                short row.  MSP_SPGEMM_SMALL=0 disables (the
+                                v5 behaviour: one too-wide row sends every
+                                short row to the ESC tiles). */
+    int64_t bitmap_rows;     /* short rows taking the bitmap / hash path */
 } msp_spgemm_info;
 
 msp_status msp_spgemm_setup_workspace(const msp_csr *A, const msp_csr *B, size_t *bytes);

@@ -48,7 +48,8 @@ class msp_spgemm_info(ctypes.Structure):
                 ("long_products", ctypes.c_int64), ("max_row_products", ctypes.c_int64),
                 ("main_ws_bytes", ctypes.c_int64), ("long_chunks", ctypes.c_int64),
                 ("max_tile_span", ctypes.c_int64), ("segmented_rows", ctypes.c_int64),
-                ("row_accumulator", ctypes.c_int64)]
+                ("row_accumulator", ctypes.c_int64), ("small_rows", ctypes.c_int64),
+                ("bitmap_rows", ctypes.c_int64)]
 
 
 _P = ctypes.POINTER

@@ -66,6 +66,9 @@ msp_status scan_nonempty_rows(const int32_t *rp, int64_t m, int64_t *pos, void *
 // S[j] = sum_{k<j} (Brp[Acol[k]+1] - Brp[Acol[k]]), j in [0, nnzA] (SpGEMM setup)
 msp_status scan_widths_to_S(const int32_t *Acol, const int32_t *Brp, int64_t nnzA, int64_t *S, void *ws,
                             size_t ws_bytes, cudaStream_t s);
+// the same, also recording bstart[j] = Brp[Acol[j]] (the B row each A nonzero expands)
+msp_status scan_widths_to_S_bstart(const int32_t *Acol, const int32_t *Brp, int64_t nnzA, int64_t *S, int32_t *bstart,
+                                   void *ws, size_t ws_bytes, cudaStream_t s);
 
 // ---------------------------------------------------------------- ops ----
 size_t spmv_ws_bytes(const msp_csr *A);

@@ -37,6 +37,17 @@ struct LoadWidth {  // nnz of the B row referenced by A nonzero i
         return int64_t(__ldg(brp + k + 1)) - __ldg(brp + k);
     }
 };
+struct LoadWidthStart {  // as LoadWidth, and records the B row start of A nonzero i
+    const int32_t *acol, *brp;
+    int32_t *bstart;
+    __device__ int64_t operator()(int64_t i) const
+    {
+        const int32_t k = acol[i];
+        const int32_t b0 = __ldg(brp + k);
+        bstart[i] = b0;
+        return int64_t(__ldg(brp + k + 1)) - b0;
+    }
+};
 struct LoadNonEmpty {  // 1 if row i has nonzeros
     const int32_t *rp;
     __device__ int64_t operator()(int64_t i) const { return __ldg(rp + i + 1) > __ldg(rp + i) ? 1 : 0; }
@@ -174,6 +185,13 @@ msp_status run_scan(In in, Out out, int64_t n, int64_t *total, int64_t *out0_if_
 size_t scan_ws_bytes(int64_t n)
 {
     return 512 + size_t(ceil_div(n > 0 ? n : 1, SCAN_TILE)) * 8 + 256;
+}
+
+msp_status scan_widths_to_S_bstart(const int32_t *Acol, const int32_t *Brp, int64_t nnzA, int64_t *S, int32_t *bstart,
+                                   void *ws, size_t ws_bytes, cudaStream_t s)
+{
+    return run_scan<LoadWidthStart, StoreI64, true>(LoadWidthStart{Acol, Brp, bstart}, StoreI64{S}, nnzA, nullptr, S,
+                                                    ws, ws_bytes, s);
 }
 
 msp_status scan_i32_to_i64(const int32_t *in, int64_t *out, int64_t n, void *ws, size_t ws_bytes, cudaStream_t s)

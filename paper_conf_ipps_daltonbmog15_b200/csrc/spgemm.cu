@@ -305,41 +305,338 @@ __device__ __forceinline__ int warp_excl_sum(int v, int lane, int *total)
     return inc - v;
 }
 
-// Span of every short row with products (warp per row); counts the short
-// rows whose span exceeds WR_SPAN into *fail.
-__global__ void wr_span_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
-                               const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
-                               const uint8_t *__restrict__ rowlong, int32_t *__restrict__ lo_out,
-                               int32_t *__restrict__ hi_out, unsigned long long *__restrict__ fail)
+// Short-row modes of the warp-row path (wmode[r]).  WM_NONE: long, or no
+// products (C.row_offsets is cleared before symbolic, so nothing to do);
+// WM_BITMAP: the bitmap / hash accumulator below (output span <= WR_SPAN);
+// WM_SMALL: the compare-count path (ws_small_kernel).
+enum : uint8_t { WM_NONE = 0, WM_BITMAP = 1, WM_SMALL = 2 };
+constexpr int WS_ALWAYS = 64;    // rows with at most this many products take the small path
+constexpr int WS_PMAX = 256;     // ... and wider-than-WR_SPAN rows with at most this many
+constexpr int WS_BATCH = 256;    // products (and A nonzeros) per warp batch of small rows
+constexpr int WS_PPL = WS_BATCH / 32;
+
+// Row classification for the warp-row path, 32 rows per warp round (lane per
+// row): P_r = S[rp[r+1]] - S[rp[r]], nnz_r = rp[r+1] - rp[r].  Rows with
+// 1 <= P_r <= WS_ALWAYS (and nnz_r <= WS_BATCH) are SMALL without a span;
+// the others get their output span (warp-cooperative, one row at a time):
+// span <= WR_SPAN -> BITMAP; wider and P_r, nnz_r <= WS_PMAX -> SMALL;
+// wider still -> promoted to a long row (rowlong / longflag set: the global
+// phase takes it).  With the small path off (MSP_SPGEMM_SMALL=0, the v5
+// behaviour) every row with products needs the bitmap and a too-wide one is
+// counted in stats[7], which turns the warp-row path off.  stats: [7]
+// too-wide rows (small path off), [8] widest BITMAP span, [9] SMALL rows,
+// [10] BITMAP rows, [11] rows promoted to long.
+__global__ void wr_class_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
+                                const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
+                                const int64_t *__restrict__ S, uint8_t *__restrict__ rowlong,
+                                int32_t *__restrict__ longflag, int32_t *__restrict__ lo_out,
+                                int32_t *__restrict__ hi_out, uint8_t *__restrict__ wmode,
+                                unsigned long long *__restrict__ stats, int small_on)
 {
     const int lane = threadIdx.x & 31;
     const int64_t nwarps = int64_t(gridDim.x) * (blockDim.x >> 5);
-    unsigned long long nfail = 0, mxspan = 0;
-    for (int64_t r = int64_t(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5); r < m; r += nwarps) {
-        if (rowlong[r]) continue;
-        const int32_t a0 = Arp[r], a1 = Arp[r + 1];
-        int32_t lo = INT_MAX, hi = -1;
-        for (int32_t j = a0 + lane; j < a1; j += 32) {
-            const int32_t k = Acol[j], b0 = Brp[k], b1 = Brp[k + 1];
-            if (b1 > b0) {
-                lo = min(lo, Bcol[b0]);
-                hi = max(hi, Bcol[b1 - 1]);
+    unsigned long long nwide = 0, mxspan = 0, nsmall = 0, nbitmap = 0, npromo = 0;
+    for (int64_t r0 = (int64_t(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5)) * 32; r0 < m;
+         r0 += nwarps * 32) {
+        const int64_t r = r0 + lane;
+        int mode = WM_NONE;
+        int32_t a0 = 0, a1 = 0;
+        bool need = false, fit = false;
+        if (r < m && !rowlong[r]) {
+            a0 = Arp[r];
+            a1 = Arp[r + 1];
+            const int64_t P = S[a1] - S[a0];
+            fit = small_on && P <= WS_PMAX && a1 - a0 <= WS_BATCH;
+            if (P > 0) {
+                if (fit && P <= WS_ALWAYS) mode = WM_SMALL;
+                else need = true;
             }
         }
-        lo = __reduce_min_sync(0xffffffffu, lo);
-        hi = __reduce_max_sync(0xffffffffu, hi);
-        if (lane == 0) {
-            lo_out[r] = lo;
-            hi_out[r] = hi;
-            if (hi >= lo) {
-                const unsigned long long sp = (unsigned long long)(int64_t(hi) - lo + 1);
-                if (sp > WR_SPAN) ++nfail;
-                mxspan = sp > mxspan ? sp : mxspan;
+        unsigned nb = __ballot_sync(0xffffffffu, need);
+        while (nb) {
+            const int src = __ffs(nb) - 1;
+            nb &= nb - 1;
+            const int32_t b_a0 = __shfl_sync(0xffffffffu, a0, src), b_a1 = __shfl_sync(0xffffffffu, a1, src);
+            int32_t lo = INT_MAX, hi = -1;
+            for (int32_t j = b_a0 + lane; j < b_a1; j += 32) {
+                const int32_t k = Acol[j], b0 = Brp[k], b1 = Brp[k + 1];
+                if (b1 > b0) {
+                    lo = min(lo, Bcol[b0]);
+                    hi = max(hi, Bcol[b1 - 1]);
+                }
             }
+            lo = __reduce_min_sync(0xffffffffu, lo);
+            hi = __reduce_max_sync(0xffffffffu, hi);
+            if (lane == src) {
+                lo_out[r] = lo;
+                hi_out[r] = hi;
+                const unsigned long long sp = (unsigned long long)(int64_t(hi) - lo + 1);
+                if (sp <= WR_SPAN) {
+                    mode = WM_BITMAP;
+                    mxspan = sp > mxspan ? sp : mxspan;
+                } else if (fit) {
+                    mode = WM_SMALL;
+                } else if (small_on) {
+                    rowlong[r] = 1;
+                    longflag[r] = 1;
+                    ++npromo;
+                } else {
+                    ++nwide;
+                }
+            }
+        }
+        if (r < m) wmode[r] = uint8_t(mode);
+        nsmall += mode == WM_SMALL;
+        nbitmap += mode == WM_BITMAP;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        nwide += __shfl_xor_sync(0xffffffffu, nwide, o);
+        mxspan = max(mxspan, __shfl_xor_sync(0xffffffffu, mxspan, o));
+        nsmall += __shfl_xor_sync(0xffffffffu, nsmall, o);
+        nbitmap += __shfl_xor_sync(0xffffffffu, nbitmap, o);
+        npromo += __shfl_xor_sync(0xffffffffu, npromo, o);
+    }
+    if (lane == 0) {
+        if (nwide) atomicAdd(stats + 7, nwide);
+        if (mxspan) atomicMax(stats + 8, mxspan);
+        if (nsmall) atomicAdd(stats + 9, nsmall);
+        if (nbitmap) atomicAdd(stats + 10, nbitmap);
+        if (npromo) atomicAdd(stats + 11, npromo);
+    }
+}
+
+// ------------------------------------------------ small rows (warp sort)
+// Rows with few products (C5's random rows: ~16; the uniform rows of C4) are
+// too small for a warp each and too wide for a bitmap.  A warp takes 32 rows
+// at a time (lane per row: mode, offsets) and processes runs of consecutive
+// SMALL rows with at most WS_BATCH products and A nonzeros together -- ESC
+// with the warp as the tile and the registers as the sort
+// buffer:
+//   A: lane per A nonzero j -- B row start (setup's bstart[j]) and product
+//      offset S[j] into shared memory (and a_ij, numeric);
+//   B: expansion, lane per product p (WS_PPL per lane, strided, all gathers
+//      in flight together): a search over the staged offsets finds p's A
+//      nonzero; the B column (and the fp64 product a_ik * b_kj, one rounding)
+//      lands at p in shared memory.  Positions follow Gustavson's order
+//      (k ascending, then B's order);
+//   C: compression, lane per product p of row r (segment [s_r, e_r) of the
+//      batch; rounds of 32 consecutive positions, each lane looping over its
+//      own row only).  p is the FIRST occurrence of its column c iff no q in
+//      [s_r, p) holds c; symbolic counts the first occurrences per row.
+//      Numeric: a row whose C row length equals P_r has no duplicates and
+//      p's rank is the number of smaller columns in the segment; otherwise
+//      first occurrences are marked (sign bit), each computes its rank among
+//      the marked columns and sums the products of c in position order
+//      (= k order: the oracle's order, separate roundings).  (c, sum) goes
+//      to C.rp[r] + rank.
+// O(P_r) work per product: fewer instructions than sorting the batch (a
+// 256-key bitonic network in registers measured 44 G warp instructions on
+// C5 symbolic vs the loops' fraction of that), no global
+// scratch, no atomics outside shared memory.
+constexpr int WS_WARPS = 4;
+template <typename V, bool NUM>
+__global__ void __launch_bounds__(WS_WARPS * 32, 8)
+ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const V *__restrict__ Aval,
+                const int32_t *__restrict__ bstart, const int32_t *__restrict__ Bcol, const V *__restrict__ Bval,
+                const uint8_t *__restrict__ wmode, const int64_t *__restrict__ S, int32_t *__restrict__ Crp,
+                int32_t *__restrict__ Ccol, V *__restrict__ Cval)
+{
+    constexpr unsigned FULL = 0xffffffffu;
+    __shared__ __align__(16) int32_t s_key_all[WS_WARPS][WS_BATCH];  // B: column by position
+    __shared__ int32_t s_b0_all[WS_WARPS][WS_BATCH];                 // A: B row start; D: head prefix H
+    __shared__ int16_t s_off_all[WS_WARPS][WS_BATCH + 2];            // A: product offset; D: sorted position | head
+    __shared__ unsigned s_first_all[NUM ? WS_WARPS : 1][WS_BATCH / 32];     // C: first-occurrence bits
+    __shared__ int s_cnt_all[WS_WARPS][32];                                   // C: symbolic row counts
+    __shared__ double s_val_all[NUM ? WS_WARPS : 1][NUM ? WS_BATCH : 1];
+    __shared__ double s_av_all[NUM ? WS_WARPS : 1][NUM ? WS_BATCH : 1];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    int32_t *s_key = s_key_all[warp];
+    int32_t *s_b0 = s_b0_all[warp];
+    int16_t *s_off = s_off_all[warp];
+    unsigned *s_first = s_first_all[NUM ? warp : 0];
+    int *s_cnt = s_cnt_all[warp];
+    double *s_val = s_val_all[NUM ? warp : 0];
+    double *s_av = s_av_all[NUM ? warp : 0];
+    const int64_t nwarps = int64_t(gridDim.x) * WS_WARPS;
+    s_cnt[lane] = 0;
+    for (int64_t r0 = (int64_t(blockIdx.x) * WS_WARPS + warp) * 32; r0 < m; r0 += nwarps * 32) {
+        const int64_t r = r0 + lane;
+        bool sm = false;
+        int32_t a0 = 0, a1 = 0, cb = 0;
+        int64_t p0 = 0;
+        int P = 0, U = 0;
+        if (r < m && wmode[r] == WM_SMALL) {
+            sm = true;
+            a0 = Arp[r];
+            a1 = Arp[r + 1];
+            p0 = S[a0];
+            P = int(S[a1] - p0);
+            if (NUM) {
+                cb = Crp[r];
+                U = Crp[r + 1] - cb;  // == P: no duplicate columns in the row
+            }
+        }
+        unsigned todo = __ballot_sync(FULL, sm);
+        while (todo) {
+            // batch: the run of consecutive SMALL lanes from s whose products
+            // and A nonzeros fit
+            const int s = __ffs(todo) - 1;
+            const int64_t base = __shfl_sync(FULL, p0, s);
+            const int32_t ja = __shfl_sync(FULL, a0, s);
+            const bool fits = sm && lane >= s && (p0 + P - base) <= WS_BATCH && a1 - ja <= WS_BATCH;
+            const unsigned fm = __ballot_sync(FULL, fits) >> s;
+            const int run = (~fm) ? __ffs(~fm) - 1 : 32 - s;
+            const int e = s + run;  // lanes [s, e)
+            todo &= ~unsigned(((1ull << run) - 1ull) << s);
+            const int32_t jb = __shfl_sync(FULL, a1, e - 1);
+            const int na = jb - ja;
+            const int np = int(__shfl_sync(FULL, p0, e - 1) - base) + __shfl_sync(FULL, P, e - 1);
+            const int prel = int(p0 - base);  // this lane's row start in the batch (lanes in [s, e))
+            const bool inb = lane >= s && lane < e;
+            // ---- A: stage the batch's A nonzeros ----
+#pragma unroll
+            for (int u = 0; u < WS_PPL; ++u) {
+                const int i = u * 32 + lane;
+                if (i < na) {
+                    const int32_t j = ja + i;
+                    s_b0[i] = bstart[j];
+                    s_off[i] = int16_t(S[j] - base);
+                    if constexpr (NUM) s_av[i] = double(Aval[j]);
+                }
+            }
+            __syncwarp();
+            // ---- B: expand (all WS_PPL gathers of a lane in flight) ----
+            int pa[WS_PPL];  // A nonzero (batch index) of product u*32 + lane
+#pragma unroll
+            for (int u = 0; u < WS_PPL; ++u) pa[u] = 0;
+#pragma unroll
+            for (int stp = WS_BATCH / 2; stp >= 1; stp >>= 1) {
+                if (stp < na) {
+#pragma unroll
+                    for (int u = 0; u < WS_PPL; ++u) {
+                        const int c = pa[u] + stp;
+                        if (c < na && s_off[c] <= u * 32 + lane) pa[u] = c;
+                    }
+                }
+            }
+            {
+                int32_t ck[WS_PPL];
+                double cv[WS_PPL];
+#pragma unroll
+                for (int u = 0; u < WS_PPL; ++u) {
+                    const int p = u * 32 + lane;
+                    ck[u] = 0;
+                    cv[u] = 0.0;
+                    if (p < np) {
+                        const int32_t bi = s_b0[pa[u]] + (p - s_off[pa[u]]);
+                        ck[u] = Bcol[bi];
+                        if constexpr (NUM) cv[u] = __dmul_rn(s_av[pa[u]], double(Bval[bi]));
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < WS_PPL; ++u) {
+                    const int p = u * 32 + lane;
+                    if (p < np) {
+                        s_key[p] = ck[u];
+                        if constexpr (NUM) s_val[p] = cv[u];
+                    }
+                }
+            }
+            __syncwarp();
+            // ---- C: compression, lane per product, rounds of 32 positions ----
+            for (int pr = 0; pr < np; pr += 32) {
+                const int p = pr + lane;
+                int t = s;  // the product's row lane: last lane in [s, e) starting at or before p
+#pragma unroll
+                for (int stp = 16; stp >= 1; stp >>= 1) {
+                    const int c = t + stp;
+                    const int oc = __shfl_sync(FULL, prel, c & 31);
+                    if (c < e && oc <= p) t = c;
+                }
+                const int seg = __shfl_sync(FULL, prel, t);
+                const int len = __shfl_sync(FULL, P, t);
+                const int32_t rowc = __shfl_sync(FULL, cb, t);
+                const bool act = p < np;
+                const int32_t c = act ? s_key[p] : 0;
+                if constexpr (!NUM) {
+                    bool first = act;
+                    for (int q = seg; q < p; ++q) first = first && (s_key[q] != c);
+                    if (first) atomicAdd(&s_cnt[t], 1);
+                } else {
+                    const bool dupfree = __shfl_sync(FULL, U, t) == len;
+                    if (act && dupfree) {
+                        int rk = 0;
+                        for (int q = seg; q < seg + len; ++q) rk += s_key[q] < c ? 1 : 0;
+                        Ccol[rowc + rk] = c;
+                        Cval[rowc + rk] = V(s_val[p]);
+                    }
+                }
+            }
+            if constexpr (NUM) {
+                // rows with duplicate columns: mark first occurrences, then rank
+                // among marked columns and sum each column's run in order
+                const bool anydup = __any_sync(FULL, inb && U != P);
+                if (anydup) {
+                    __syncwarp();
+                    for (int pr = 0; pr < np; pr += 32) {
+                        const int p = pr + lane;
+                        int t = s;
+#pragma unroll
+                        for (int stp = 16; stp >= 1; stp >>= 1) {
+                            const int c = t + stp;
+                            const int oc = __shfl_sync(FULL, prel, c & 31);
+                            if (c < e && oc <= p) t = c;
+                        }
+                        const int seg = __shfl_sync(FULL, prel, t);
+                        const bool dup = __shfl_sync(FULL, U, t) != __shfl_sync(FULL, P, t);
+                        bool first = false;
+                        if (p < np && dup) {
+                            const int32_t c = s_key[p];
+                            first = true;
+                            for (int q = seg; q < p; ++q) first = first && (s_key[q] != c);
+                        }
+                        s_first[pr / 32] = __ballot_sync(FULL, first);  // one word per round
+                    }
+                    __syncwarp();
+                    for (int pr = 0; pr < np; pr += 32) {
+                        const int p = pr + lane;
+                        int t = s;
+#pragma unroll
+                        for (int stp = 16; stp >= 1; stp >>= 1) {
+                            const int c = t + stp;
+                            const int oc = __shfl_sync(FULL, prel, c & 31);
+                            if (c < e && oc <= p) t = c;
+                        }
+                        const int seg = __shfl_sync(FULL, prel, t);
+                        const int len = __shfl_sync(FULL, P, t);
+                        const int32_t rowc = __shfl_sync(FULL, cb, t);
+                        const bool dup = __shfl_sync(FULL, U, t) != len;
+                        if (p < np && dup && ((s_first[pr / 32] >> lane) & 1u)) {
+                            const int32_t c = s_key[p];
+                            int rk = 0;
+                            double sum = s_val[p];
+                            for (int q = seg; q < seg + len; ++q) {
+                                const int32_t kq = s_key[q];
+                                const bool fq = (s_first[q >> 5] >> (q & 31)) & 1u;
+                                rk += (fq && kq < c) ? 1 : 0;
+                                if (kq == c && q > p) sum = __dadd_rn(sum, s_val[q]);
+                            }
+                            Ccol[rowc + rk] = c;
+                            Cval[rowc + rk] = V(sum);
+                        }
+                    }
+                }
+            }
+            __syncwarp();
+        }
+        if constexpr (!NUM) {
+            __syncwarp();
+            if (sm) Crp[r + 1] = s_cnt[lane];  // Crp holds the row offsets: row r's count goes to Crp[r + 1]
+            s_cnt[lane] = 0;
+            __syncwarp();
         }
     }
-    if (lane == 0 && nfail) atomicAdd(fail, nfail);
-    if (lane == 0 && mxspan) atomicMax(fail + 1, mxspan);
 }
 
 // One step per A nonzero of a chunk of <= 32 (lane l holds nonzero l's B
@@ -407,7 +704,7 @@ __device__ __forceinline__ int nth_set_bit(uint32_t w, int n)
 __global__ void __launch_bounds__(WR_SYM_WARPS * 32, 1)
 wr_symbolic_kernel(int32_t m, int nw_max, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
                    const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
-                   const uint8_t *__restrict__ rowlong, const int64_t *__restrict__ S,
+                   const uint8_t *__restrict__ wmode, const int64_t *__restrict__ S,
                    const int32_t *__restrict__ spanlo, const int32_t *__restrict__ spanhi,
                    int32_t *__restrict__ Crp_counts, int32_t *__restrict__ ucol)
 {
@@ -416,12 +713,8 @@ wr_symbolic_kernel(int32_t m, int nw_max, const int32_t *__restrict__ Arp, const
     uint32_t *bm = wr_bm_all + size_t(warp) * nw_max;  // nw_max: a multiple of 128 words
     const int64_t nwarps = int64_t(gridDim.x) * WR_SYM_WARPS;
     for (int64_t r = int64_t(blockIdx.x) * WR_SYM_WARPS + warp; r < m; r += nwarps) {
-        if (rowlong[r]) continue;
+        if (wmode[r] != WM_BITMAP) continue;  // long, small or without products (counts cleared)
         const int32_t lo = spanlo[r], hi = spanhi[r];
-        if (hi < lo) {  // no products
-            if (lane == 0) Crp_counts[r] = 0;
-            continue;
-        }
         const int nw = (hi - lo + 32) >> 5;
         const int nq = (nw + 127) >> 7;  // rounds of 4 words per lane
         for (int q = 0; q < nq; ++q) reinterpret_cast<uint4 *>(bm)[q * 32 + lane] = make_uint4(0u, 0u, 0u, 0u);
@@ -496,7 +789,7 @@ template <typename V>
 __global__ void __launch_bounds__(WR_NUM_WARPS * 32, 3)
 wr_numeric_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
                   const V *__restrict__ Aval, const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
-                  const V *__restrict__ Bval, const uint8_t *__restrict__ rowlong, const int64_t *__restrict__ S,
+                  const V *__restrict__ Bval, const uint8_t *__restrict__ wmode, const int64_t *__restrict__ S,
                   const int32_t *__restrict__ spanlo, const int32_t *__restrict__ ucol,
                   const int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol, V *__restrict__ Cval)
 {
@@ -514,7 +807,7 @@ wr_numeric_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
     auto load_hdr = [&](int64_t rr) {
         Hdr h{0, 0, 0, 0, 0, 1};
         if (rr < m) {
-            h.skip = rowlong[rr];
+            h.skip = wmode[rr] != WM_BITMAP;
             h.cb = Crp[rr];
             h.ce = Crp[rr + 1];
             h.a0 = Arp[rr];
@@ -631,11 +924,14 @@ struct SetupWs {
     int64_t *longC;      // [m]  chunks of the i-th long row
     int64_t *longCO;     // [m + 1] prefix of longC
     unsigned long long *stats;  // [16]: [0] max row products, [1..6] gathered setup sizes, [7] short rows
-                                //       too wide for the row accumulator, [8] widest short-row span
+                                //       too wide for the row accumulator (small path off), [8] widest
+                                //       BITMAP span, [9] SMALL rows, [10] BITMAP rows, [11] promoted rows
     int32_t *spanlo, *spanhi;   // [m] output column span of each long row (segmented path, f3)
     int32_t *spaflag;           // [m] 1 = the row takes the segmented path
     int64_t *spapos;            // [m + 1]
     int32_t *sparow;            // [m] rows of the segmented path
+    int32_t *bstart;            // [nnzA] B row start of each A nonzero (Brp[Acol[j]])
+    uint8_t *wmode;             // [m] warp-row path mode of each short row (WM_*)
     void *scan;
     size_t scan_bytes;
     size_t bytes;
@@ -662,6 +958,8 @@ SetupWs carve_setup(const msp_csr *A, void *ws, size_t cap, bool *ok)
     w.spaflag = cv.take<int32_t>(size_t(m > 0 ? m : 1));
     w.spapos = cv.take<int64_t>(size_t(m + 1));
     w.sparow = cv.take<int32_t>(size_t(m > 0 ? m : 1));
+    w.bstart = cv.take<int32_t>(size_t(nnz > 0 ? nnz : 1));
+    w.wmode = cv.take<uint8_t>(size_t(m > 0 ? m : 1));
     w.scan_bytes = scan_ws_bytes(std::max<int64_t>(std::max<int64_t>(m, nnz), 1));
     w.scan = cv.take<char>(w.scan_bytes);
     w.bytes = cv.off;
@@ -1312,7 +1610,7 @@ MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, int64_t nucol, void *ws
 }
 
 struct HostInfo {  // read back by setup (one synchronisation), passed to symbolic / numeric in msp_spgemm_info
-    int64_t nprods, nlong, LP, LC, maxP, nspa, rowacc;
+    int64_t nprods, nlong, LP, LC, maxP, nspa, rowacc, nsmall, nbitmap;
 };
 
 // The setup sizes gathered into one device array (so setup reads them back
@@ -1331,15 +1629,15 @@ __global__ void info_gather_kernel(const int64_t *__restrict__ S, int64_t nnzA, 
     out[3] = nlong > 0 ? longCO[nlong] : 0;
     out[4] = int64_t(stats[0]);
     out[5] = spapos[m];
-    // out[6], out[7] are stats[7], stats[8] themselves: short rows too wide for
-    // the row accumulator, widest short-row span
+    // out[6..9] are stats[7..10] themselves: short rows too wide for the row
+    // accumulator, widest BITMAP span, SMALL rows, BITMAP rows
 }
 
 // A pinned host staging word array per host thread for the synchronising reads.
 int64_t *pinned_words()
 {
     static thread_local int64_t *p = nullptr;
-    if (!p && cudaMallocHost(reinterpret_cast<void **>(&p), 8 * sizeof(int64_t)) != cudaSuccess) p = nullptr;
+    if (!p && cudaMallocHost(reinterpret_cast<void **>(&p), 16 * sizeof(int64_t)) != cudaSuccess) p = nullptr;
     return p;
 }
 
@@ -1354,6 +1652,7 @@ msp_status read_back(const int64_t *dev, int n, int64_t *host, cudaStream_t s, c
 }
 
 bool rowacc_enabled();
+bool small_enabled();
 
 msp_status read_info(const SetupWs &sw, int64_t m, int64_t nnzA, HostInfo *h, cudaStream_t s)
 {
@@ -1361,8 +1660,8 @@ msp_status read_info(const SetupWs &sw, int64_t m, int64_t nnzA, HostInfo *h, cu
                                         reinterpret_cast<int64_t *>(sw.stats) + 1);
     msp_status st = last_launch("info_gather_kernel");
     if (st != MSP_OK) return st;
-    int64_t v[8];
-    st = read_back(reinterpret_cast<const int64_t *>(sw.stats) + 1, 8, v, s, "spgemm: setup sizes");
+    int64_t v[10];
+    st = read_back(reinterpret_cast<const int64_t *>(sw.stats) + 1, 10, v, s, "spgemm: setup sizes");
     if (st != MSP_OK) return st;
     h->nprods = v[0];
     h->nlong = v[1];
@@ -1370,8 +1669,10 @@ msp_status read_info(const SetupWs &sw, int64_t m, int64_t nnzA, HostInfo *h, cu
     h->LC = v[3];
     h->maxP = v[4];
     h->nspa = v[5];
-    // row accumulator: 0 = off, else the widest short-row span (sizes the bitmaps)
+    // warp-row path: 0 = off (ESC tiles), else the widest BITMAP span, at least 1 (sizes the bitmaps)
     h->rowacc = (rowacc_enabled() && v[6] == 0) ? std::max<int64_t>(v[7], 1) : 0;
+    h->nsmall = h->rowacc ? v[8] : 0;
+    h->nbitmap = h->rowacc ? v[9] : 0;
     return MSP_OK;
 }
 
@@ -1456,14 +1757,47 @@ bool rowacc_enabled()
     return v != 0;
 }
 
+bool small_enabled()
+{
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("MSP_SPGEMM_SMALL");  // 0: no compare-count path (round-2 behaviour, ablation)
+        v = (e && atoi(e) == 0) ? 0 : 1;
+    }
+    return v != 0;
+}
+
+template <typename V, bool NUM>
+msp_status run_small(const msp_csr *A, const msp_csr *B, const SetupWs &sw, int32_t *Crp, int32_t *Ccol, void *Cval,
+                     cudaStream_t s)
+{
+    auto kern = ws_small_kernel<V, NUM>;
+    int occ = 1;
+    msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), 0, "spgemm: small rows", WS_WARPS * 32, &occ,
+                                  true);
+    if (st != MSP_OK) return st;
+    const int32_t m = A->nrows;
+    const int64_t g = std::min<int64_t>(int64_t(occ) * sm_count(), ceil_div(m, WS_WARPS * 32));
+    kern<<<unsigned(g > 0 ? g : 1), WS_WARPS * 32, 0, s>>>(m, A->row_offsets, static_cast<const V *>(A->vals),
+                                                          sw.bstart, B->col_idx, static_cast<const V *>(B->vals),
+                                                          sw.wmode, sw.S, Crp, Ccol, static_cast<V *>(Cval));
+    return last_launch(NUM ? "ws_small_kernel<numeric>" : "ws_small_kernel<symbolic>");
+}
+
 template <bool NUM>
-msp_status run_rowacc(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, int64_t rowacc_span,
+msp_status run_rowacc(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, const HostInfo &h,
                       int32_t *Crp, int32_t *Ccol, void *Cval, cudaStream_t s)
 {
     const int32_t m = A->nrows;
+    if (h.nsmall > 0) {
+        msp_status st = (A->dtype == MSP_F64) ? run_small<double, NUM>(A, B, sw, Crp, Ccol, Cval, s)
+                                              : run_small<float, NUM>(A, B, sw, Crp, Ccol, Cval, s);
+        if (st != MSP_OK) return st;
+    }
+    if (h.nbitmap <= 0) return MSP_OK;
     if (!NUM) {
         // bitmap words per warp: the widest short row's span, in rounds of 128 words
-        const int nw_max = int(ceil_div(ceil_div(rowacc_span, 32), 128) * 128);
+        const int nw_max = int(ceil_div(ceil_div(h.rowacc, 32), 128) * 128);
         const int smem = WR_SYM_WARPS * nw_max * 4;
         // the carveout / occupancy query is per bitmap size: no per-kernel cache here
         msp_status st = cuda_check(cudaFuncSetAttribute(reinterpret_cast<const void *>(wr_symbolic_kernel),
@@ -1478,7 +1812,7 @@ msp_status run_rowacc(const msp_csr *A, const msp_csr *B, const SetupWs &sw, con
         if (occ < 1) occ = 1;
         const int64_t g = std::min<int64_t>(int64_t(occ) * sm_count(), ceil_div(m, WR_SYM_WARPS));
         wr_symbolic_kernel<<<unsigned(g > 0 ? g : 1), WR_SYM_WARPS * 32, smem, s>>>(
-            m, nw_max, A->row_offsets, A->col_idx, B->row_offsets, B->col_idx, sw.rowlong, sw.S, sw.spanlo,
+            m, nw_max, A->row_offsets, A->col_idx, B->row_offsets, B->col_idx, sw.wmode, sw.S, sw.spanlo,
             sw.spanhi, Crp + 1, mw.ucol);
         return last_launch("wr_symbolic_kernel");
     }
@@ -1491,7 +1825,7 @@ msp_status run_rowacc(const msp_csr *A, const msp_csr *B, const SetupWs &sw, con
         const int64_t g = std::min<int64_t>(int64_t(occ) * sm_count(), ceil_div(m, WR_NUM_WARPS));
         kern<<<unsigned(g > 0 ? g : 1), WR_NUM_WARPS * 32, WR_NUM_SMEM, s>>>(
             m, A->row_offsets, A->col_idx, static_cast<const double *>(A->vals), B->row_offsets, B->col_idx,
-            static_cast<const double *>(B->vals), sw.rowlong, sw.S, sw.spanlo, mw.ucol, Crp, Ccol,
+            static_cast<const double *>(B->vals), sw.wmode, sw.S, sw.spanlo, mw.ucol, Crp, Ccol,
             static_cast<double *>(Cval));
     } else {
         auto kern = wr_numeric_kernel<float>;
@@ -1502,7 +1836,7 @@ msp_status run_rowacc(const msp_csr *A, const msp_csr *B, const SetupWs &sw, con
         const int64_t g = std::min<int64_t>(int64_t(occ) * sm_count(), ceil_div(m, WR_NUM_WARPS));
         kern<<<unsigned(g > 0 ? g : 1), WR_NUM_WARPS * 32, WR_NUM_SMEM, s>>>(
             m, A->row_offsets, A->col_idx, static_cast<const float *>(A->vals), B->row_offsets, B->col_idx,
-            static_cast<const float *>(B->vals), sw.rowlong, sw.S, sw.spanlo, mw.ucol, Crp, Ccol,
+            static_cast<const float *>(B->vals), sw.wmode, sw.S, sw.spanlo, mw.ucol, Crp, Ccol,
             static_cast<float *>(Cval));
     }
     return last_launch("wr_numeric_kernel");
@@ -1547,7 +1881,8 @@ msp_status prepare_main(const msp_csr *A, const void *ws1, size_t b1, void *ws2,
     bool ok1, ok2;
     *sw = carve_setup(A, const_cast<void *>(ws1), b1, &ok1);
     if (!ok1) return MSP_ERR_WORKSPACE;
-    *mw = carve_main(A->nrows, ntiles_of(A->nnz, h.nprods, h.rowacc), h.LP, h.rowacc ? h.nprods : 0, ws2, b2, &ok2);
+    *mw = carve_main(A->nrows, ntiles_of(A->nnz, h.nprods, h.rowacc), h.LP, h.nbitmap > 0 ? h.nprods : 0, ws2, b2,
+                     &ok2);
     if (!ok2) return MSP_ERR_WORKSPACE;
     return MSP_OK;
 }
@@ -1562,6 +1897,8 @@ HostInfo host_info(const msp_spgemm_info *info)
     h.maxP = info->max_row_products;
     h.nspa = info->segmented_rows;
     h.rowacc = info->row_accumulator;
+    h.nsmall = info->small_rows;
+    h.nbitmap = info->bitmap_rows;
     return h;
 }
 
@@ -1599,7 +1936,7 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
         st = last_launch("arow_kernel");
         if (st != MSP_OK) return st;
     }
-    st = scan_widths_to_S(A->col_idx, B->row_offsets, nnz, w.S, w.scan, w.scan_bytes, s);
+    st = scan_widths_to_S_bstart(A->col_idx, B->row_offsets, nnz, w.S, w.bstart, w.scan, w.scan_bytes, s);
     if (st != MSP_OK) return st;
     if (m > 0) {
         const unsigned blocks = unsigned(std::min<int64_t>(ceil_div(m, 256), 148 * 16));
@@ -1617,11 +1954,11 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
             st = last_launch("span_kernel");
             if (st != MSP_OK) return st;
         }
-        if (nnz > 0 && rowacc_enabled()) {  // short-row spans for the row accumulator
-            wr_span_kernel<<<unsigned(std::min<int64_t>(ceil_div(m, 8), 148 * 16)), 256, 0, s>>>(
-                A->nrows, A->row_offsets, A->col_idx, B->row_offsets, B->col_idx, w.rowlong, w.spanlo, w.spanhi,
-                &w.stats[7]);  // [7] too-wide rows, [8] widest span
-            st = last_launch("wr_span_kernel");
+        if (nnz > 0 && rowacc_enabled()) {  // warp-row path: SMALL / BITMAP rows, wide rows promoted to long
+            wr_class_kernel<<<unsigned(std::min<int64_t>(ceil_div(m, 8 * 32), 148 * 16)), 256, 0, s>>>(
+                A->nrows, A->row_offsets, A->col_idx, B->row_offsets, B->col_idx, w.S, w.rowlong, w.longflag,
+                w.spanlo, w.spanhi, w.wmode, w.stats, small_enabled() ? 1 : 0);
+            st = last_launch("wr_class_kernel");
             if (st != MSP_OK) return st;
         }
         spa_classify_kernel<<<blocks, 256, 0, s>>>(A->nrows, A->row_offsets, w.S, w.spanlo, w.spanhi, w.rowlong,
@@ -1655,7 +1992,7 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
     if (st != MSP_OK) return st;
     const int64_t ntiles = ntiles_of(nnz, h.nprods, h.rowacc);
     bool ok2;
-    MainWs mw = carve_main(m, ntiles, h.LP, h.rowacc ? h.nprods : 0, nullptr, SIZE_MAX, &ok2);
+    MainWs mw = carve_main(m, ntiles, h.LP, h.nbitmap > 0 ? h.nprods : 0, nullptr, SIZE_MAX, &ok2);
     info->nprods = h.nprods;
     info->ntiles = ntiles;
     info->long_rows = h.nlong;
@@ -1666,6 +2003,8 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
     info->max_tile_span = -1;  // set by symbolic
     info->segmented_rows = h.nspa;
     info->row_accumulator = h.rowacc;
+    info->small_rows = h.nsmall;
+    info->bitmap_rows = h.nbitmap;
     return MSP_OK;
 }
 
@@ -1719,7 +2058,7 @@ msp_status spgemm_pass(const msp_csr *A, const msp_csr *B, const void *ws1, size
         return MSP_ERR_ARG;
     }
     if (h.nprods > 0 && m > 0) {
-        if (h.rowacc) st = run_rowacc<NUM>(A, B, sw, mw, h.rowacc, Crp, Ccol, Cval, s);
+        if (h.rowacc) st = run_rowacc<NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s);
         else
             st = (A->dtype == MSP_F64) ? run_tiles<double, NUM>(A, B, sw, mw, ntiles, maxspan, Crp, Ccol, Cval, s)
                                        : run_tiles<float, NUM>(A, B, sw, mw, ntiles, maxspan, Crp, Ccol, Cval, s);

@@ -27,7 +27,7 @@ def test_library_exports_every_declared_symbol():
     L = _lib.lib()
     for name in declared_symbols():
         assert hasattr(L, name), name
-    assert L.msp_version() == 5
+    assert L.msp_version() == 6
 
 
 def test_only_abi_symbols_exported():

@@ -98,9 +98,12 @@ def test_signed_zero_and_cancellation():
     assert np.array_equal(val.view(np.uint64), W.val.view(np.uint64)), (val, W.val)
 
 
+@pytest.mark.skipif(os.environ.get("MSP_SPGEMM_SMALL") != "0" and os.environ.get("MSP_SPGEMM_ROWACC") != "0",
+                    reason="with the small path on, wide rows take it (test_gpu_spgemm_small.py)")
 def test_not_taken_on_wide_rows():
-    """One short row spanning more than 65,536 columns sends every short row
-    to the ESC tile pass (the choice is global)."""
+    """Small path off (v5 behaviour): one short row spanning more than 65,536
+    columns sends every short row to the ESC tile pass (the choice is
+    global)."""
     rng = np.random.default_rng(3)
     n = 200_000
     B = gen.CSR(3, n, np.array([0, 2, 3, 4], np.int32), np.array([0, 150_000, 7, 9], np.int32), np.ones(4))
@@ -121,6 +124,7 @@ def test_esc_tile_path_suite():
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     env = dict(os.environ, MSP_SPGEMM_ROWACC="0")
     r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", *_ESC_SUITE,
-                        "tests/test_gpu_spgemm_rowacc.py::test_not_taken_on_wide_rows"],
+                        "tests/test_gpu_spgemm_rowacc.py::test_not_taken_on_wide_rows",
+                        "tests/test_gpu_fullsize.py::test_spgemm_64bit_keys"],
                        cwd=root, env=env, capture_output=True, text=True, timeout=1800)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
