@@ -78,9 +78,13 @@ struct CtaRecord {  // one per CTA in the workspace
 
 // NW worker warps of 32 lanes x K = 8 products each (one tile = NW * 256
 // merge items), plus one producer warp and one row warp.
-template <typename V, int NW_, int STAGES_, int RSLOTS_, int MINB_>
+template <typename V, int NW_, int STAGES_, int RSLOTS_, int MINB_, bool EARLY_ = false>
 struct Cfg {
     static constexpr bool ROWK = false;
+    // EARLY: a worker issues tile t+1's x gathers right after forming tile
+    // t's products (they fly during t's walk, scan and look-back) instead of
+    // after the walk
+    static constexpr bool EARLY = EARLY_;
     static constexpr int NW = NW_;
     static constexpr int K = 8;
     static constexpr int WSPAN = 32 * K;                 // products per worker warp
@@ -130,6 +134,7 @@ struct CfgK {
     static constexpr int PROD_BYTES = NW * WMAP_BYTES;
     static constexpr int MISC_BYTES = 2048;
     static constexpr int SMEM = STAGES * STAGE_BYTES + PROD_BYTES + MISC_BYTES;
+    static constexpr bool EARLY = false;
     static_assert(K % 2 == 1 && K < 32, "K odd and < 32");
 };
 
@@ -238,10 +243,19 @@ __device__ __forceinline__ void st_global_if(float *p, float v, bool pred)
                  "r"(int(pred)));
 }
 
+// The producer's wait for a free stage.  MSP_SPMV_PROD_SPIN=1 (experiment
+// builds): a plain try_wait spin instead of the suspend-hinted wait.
+#ifndef MSP_SPMV_PROD_SPIN
+#define MSP_SPMV_PROD_SPIN 0
+#endif
 __device__ __forceinline__ void mbar_wait_backoff(uint64_t *bar, uint32_t parity)
 {
+#if MSP_SPMV_PROD_SPIN
     while (!mbar_try_wait(bar, parity)) {
     }
+#else
+    mbar_wait(bar, parity);
+#endif
 }
 
 // Split search with a guess: probe the 32 consecutive rows around `g` first
@@ -760,6 +774,9 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             if (lane == 0) mbar_arrive(&empty[stage]);
             mbar_wait(&rowsrdy[rs], (t / C::RSLOTS) & 1);
             if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 13 : 12);  // lockstep + row map
+            if constexpr (C::EARLY) {
+                if (t + 1 < ntiles) a_issue(t + 1);
+            }
             // ---- walk ----
             const uint32_t *flags = reinterpret_cast<const uint32_t *>(rslots + size_t(rs) * C::RSLOT_BYTES);
             const uint16_t *rmap =
@@ -851,7 +868,9 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
             }
             // next tile's gathers fly while the previous tile's first row is finished
             if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 10 : 6);  // walked + scanned
-            if (t + 1 < ntiles) a_issue(t + 1);
+            if constexpr (!C::EARLY) {
+                if (t + 1 < ntiles) a_issue(t + 1);
+            }
             if (lane == 0 && (warp == 0 || warp == NW - 1)) TR(t, warp ? 11 : 7);  // next tile's gathers issued
             // ---- the warp's first row of tile t-1 (deferred one tile so that
             //      the look-back never waits): carry of earlier warps (nearest
@@ -927,7 +946,11 @@ template <typename V> struct Shape<V, 4> { using C = Cfg<V, 4, 2, 4, 4>; };
 template <typename V> struct Shape<V, 5> { using C = Cfg<V, 4, 2, 4, 5>; };
 template <typename V> struct Shape<V, 6> { using C = Cfg<V, 2, 2, 4, 8>; };
 template <typename V> struct Shape<V, 7> { using C = Cfg<V, 2, 2, 4, 6>; };
-constexpr int kNumShapes = 8;
+template <typename V> struct Shape<V, 8> { using C = Cfg<V, 4, 2, 4, 4, true>; };
+template <typename V> struct Shape<V, 9> { using C = Cfg<V, 2, 2, 4, 8, true>; };
+template <typename V> struct Shape<V, 10> { using C = Cfg<V, 2, 3, 4, 8, true>; };
+template <typename V> struct Shape<V, 11> { using C = Cfg<V, 2, 4, 4, 8, true>; };
+constexpr int kNumShapes = 12;
 
 template <typename V, class C>
 msp_status launch_cfg(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_bytes, cudaStream_t s)
@@ -1042,8 +1065,13 @@ msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_
         // CTAs per SM once x spills to DRAM, where more gathers in flight only
         // add DRAM contention (C5 13.0 vs 13.3 ms).
         // (profiles/r2/spmv_irregular_shapes.txt)
+        // fp32 values with x in L2 (C3): 8 CTAs/SM of 2 workers that issue
+        // tile t+1's gathers before walking tile t (C3 455 -> 419 us; fp64
+        // spills at that size: C4 keeps shape 4, 83 vs 106 us)
+        // (profiles/r2/spmv_irregular_shapes.txt)
         if (A->nrows > 0 && double(A->nnz) >= 20.0 * double(A->nrows)) shape = -1;
-        else shape = int64_t(A->ncols) * int64_t(sizeof(V)) <= l2_bytes() / 2 ? 4 : 0;
+        else if (int64_t(A->ncols) * int64_t(sizeof(V)) <= l2_bytes() / 2) shape = sizeof(V) == 4 ? 9 : 4;
+        else shape = 0;
     }
     switch (shape) {
     case -1: {
@@ -1059,6 +1087,10 @@ msp_status launch(const msp_csr *A, const void *x, void *y, void *ws, size_t ws_
     case 5: return launch_cfg<V, typename Shape<V, 5>::C>(A, x, y, ws, ws_bytes, s);
     case 6: return launch_cfg<V, typename Shape<V, 6>::C>(A, x, y, ws, ws_bytes, s);
     case 7: return launch_cfg<V, typename Shape<V, 7>::C>(A, x, y, ws, ws_bytes, s);
+    case 8: return launch_cfg<V, typename Shape<V, 8>::C>(A, x, y, ws, ws_bytes, s);
+    case 9: return launch_cfg<V, typename Shape<V, 9>::C>(A, x, y, ws, ws_bytes, s);
+    case 10: return launch_cfg<V, typename Shape<V, 10>::C>(A, x, y, ws, ws_bytes, s);
+    case 11: return launch_cfg<V, typename Shape<V, 11>::C>(A, x, y, ws, ws_bytes, s);
     default: return launch_cfg<V, typename Shape<V, 0>::C>(A, x, y, ws, ws_bytes, s);
     }
 }
