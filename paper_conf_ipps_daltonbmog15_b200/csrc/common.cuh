@@ -82,6 +82,44 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity)
     }
 }
 
+// Read-only random gathers with a 64-byte L2 fill: a miss fetches 64
+// instead of 128 DRAM bytes (tools/probe/gather_probe.py).  Used for the
+// SpGEMM B-row and B-offset gathers; MSP_L2_64B=0 (experiment builds) gives
+// plain __ldg.
+#ifndef MSP_L2_64B
+#define MSP_L2_64B 1
+#endif
+__device__ __forceinline__ int32_t ldg64(const int32_t *p)
+{
+#if MSP_L2_64B
+    int32_t v;
+    asm("ld.global.nc.L2::64B.s32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+#else
+    return __ldg(p);
+#endif
+}
+__device__ __forceinline__ float ldg64(const float *p)
+{
+#if MSP_L2_64B
+    float v;
+    asm("ld.global.nc.L2::64B.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    return v;
+#else
+    return __ldg(p);
+#endif
+}
+__device__ __forceinline__ double ldg64(const double *p)
+{
+#if MSP_L2_64B
+    double v;
+    asm("ld.global.nc.L2::64B.f64 %0, [%1];" : "=d"(v) : "l"(p));
+    return v;
+#else
+    return __ldg(p);
+#endif
+}
+
 __device__ __forceinline__ uint64_t policy_evict_first()
 {
     uint64_t p;

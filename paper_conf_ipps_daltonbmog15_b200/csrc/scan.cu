@@ -43,9 +43,9 @@ struct LoadWidthStart {  // as LoadWidth, and records the B row start of A nonze
     __device__ int64_t operator()(int64_t i) const
     {
         const int32_t k = acol[i];
-        const int32_t b0 = __ldg(brp + k);
+        const int32_t b0 = ldg64(brp + k);
         bstart[i] = b0;
-        return int64_t(__ldg(brp + k + 1)) - b0;
+        return int64_t(ldg64(brp + k + 1)) - b0;
     }
 };
 struct LoadNonEmpty {  // 1 if row i has nonzeros

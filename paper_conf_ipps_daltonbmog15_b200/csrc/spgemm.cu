@@ -81,7 +81,7 @@ __global__ void rowclass_kernel(int32_t m, const int32_t *__restrict__ rp, const
                                 uint8_t *__restrict__ rowlong, int32_t *__restrict__ longflag,
                                 int64_t *__restrict__ longP, unsigned long long *__restrict__ maxP)
 {
-    unsigned long long mx = 0;
+    unsigned long long mx = 0, nl = 0;
     for (int64_t r = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; r < m; r += int64_t(gridDim.x) * blockDim.x) {
         const int32_t a = rp[r], b = rp[r + 1];
         const int64_t P = S[b] - S[a];
@@ -90,10 +90,15 @@ __global__ void rowclass_kernel(int32_t m, const int32_t *__restrict__ rp, const
         longflag[r] = lg ? 1 : 0;
         longP[r] = 0;
         mx = max(mx, (unsigned long long)P);
+        nl += lg;
     }
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    for (int o = 16; o > 0; o >>= 1) {
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        nl += __shfl_xor_sync(0xffffffffu, nl, o);
+    }
     if ((threadIdx.x & 31) == 0 && mx) atomicMax(maxP, mx);
+    if ((threadIdx.x & 31) == 0 && nl) atomicAdd(maxP + 12, nl);  // stats[12]: long rows
 }
 
 __global__ void long_scatter_kernel(int32_t m, const int32_t *__restrict__ rp, const int64_t *__restrict__ S,
@@ -125,9 +130,13 @@ __global__ void long_scatter_kernel(int32_t m, const int32_t *__restrict__ rp, c
 constexpr int SPA_W = 12288;    // accumulator columns (96 KB fp64 + a bit per column)
 constexpr int SPA_NT = 256;
 
-__global__ void span_init_kernel(int32_t m, int32_t *__restrict__ lo, int32_t *__restrict__ hi)
+// (long rows only: the warp-row path's classification has written the
+// BITMAP rows' spans already)
+__global__ void span_init_kernel(int32_t m, const uint8_t *__restrict__ rowlong, int32_t *__restrict__ lo,
+                                 int32_t *__restrict__ hi)
 {
     for (int64_t r = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; r < m; r += int64_t(gridDim.x) * blockDim.x) {
+        if (!rowlong[r]) continue;
         lo[r] = INT_MAX;
         hi[r] = -1;
     }
@@ -530,8 +539,8 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const V *__restrict_
                     cv[u] = 0.0;
                     if (p < np) {
                         const int32_t bi = s_b0[pa[u]] + (p - s_off[pa[u]]);
-                        ck[u] = Bcol[bi];
-                        if constexpr (NUM) cv[u] = __dmul_rn(s_av[pa[u]], double(Bval[bi]));
+                        ck[u] = ldg64(Bcol + bi);
+                        if constexpr (NUM) cv[u] = __dmul_rn(s_av[pa[u]], double(ldg64(Bval + bi)));
                     }
                 }
 #pragma unroll
@@ -1944,21 +1953,37 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
                                                w.stats);
         st = last_launch("rowclass_kernel");
         if (st != MSP_OK) return st;
+        if (nnz > 0 && rowacc_enabled()) {  // warp-row path: SMALL / BITMAP rows, wide rows promoted to long
+            wr_class_kernel<<<unsigned(std::min<int64_t>(ceil_div(m, 8 * 32), 148 * 16)), 256, 0, s>>>(
+                A->nrows, A->row_offsets, A->col_idx, B->row_offsets, B->col_idx, w.S, w.rowlong, w.longflag,
+                w.spanlo, w.spanhi, w.wmode, w.stats, small_enabled() ? 1 : 0);
+            st = last_launch("wr_class_kernel");
+            if (st != MSP_OK) return st;
+        }
+        // Large matrices: one extra synchronisation reads the long-row count
+        // (from the classification and the promotions); without long rows the
+        // global-phase bookkeeping (spans, segmented classification, four
+        // row scans, scatters) is skipped -- C5: ~4.7 ms of setup.
+        bool any_long = true;
+        if (m >= (1 << 20)) {
+            int64_t v[13];
+            st = read_back(reinterpret_cast<const int64_t *>(w.stats), 13, v, s, "spgemm: long rows");
+            if (st != MSP_OK) return st;
+            any_long = (v[11] + v[12]) > 0;
+        }
+        if (!any_long) {
+            st = cuda_check(cudaMemsetAsync(w.longpos + m, 0, sizeof(int64_t), s), "spgemm: clear");
+            if (st == MSP_OK) st = cuda_check(cudaMemsetAsync(w.spapos + m, 0, sizeof(int64_t), s), "spgemm: clear");
+            if (st != MSP_OK) return st;
+        } else {
         // segmented path for long rows with a narrow output span (f3)
-        span_init_kernel<<<blocks, 256, 0, s>>>(A->nrows, w.spanlo, w.spanhi);
+        span_init_kernel<<<blocks, 256, 0, s>>>(A->nrows, w.rowlong, w.spanlo, w.spanhi);
         st = last_launch("span_init_kernel");
         if (st != MSP_OK) return st;
         if (nnz > 0 && spa_enabled()) {
             span_kernel<<<unsigned(std::min<int64_t>(ceil_div(nnz, 256), 148 * 16)), 256, 0, s>>>(
                 nnz, A->col_idx, w.arow, w.rowlong, B->row_offsets, B->col_idx, w.spanlo, w.spanhi);
             st = last_launch("span_kernel");
-            if (st != MSP_OK) return st;
-        }
-        if (nnz > 0 && rowacc_enabled()) {  // warp-row path: SMALL / BITMAP rows, wide rows promoted to long
-            wr_class_kernel<<<unsigned(std::min<int64_t>(ceil_div(m, 8 * 32), 148 * 16)), 256, 0, s>>>(
-                A->nrows, A->row_offsets, A->col_idx, B->row_offsets, B->col_idx, w.S, w.rowlong, w.longflag,
-                w.spanlo, w.spanhi, w.wmode, w.stats, small_enabled() ? 1 : 0);
-            st = last_launch("wr_class_kernel");
             if (st != MSP_OK) return st;
         }
         spa_classify_kernel<<<blocks, 256, 0, s>>>(A->nrows, A->row_offsets, w.S, w.spanlo, w.spanhi, w.rowlong,
@@ -1982,6 +2007,7 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
         if (st != MSP_OK) return st;
         st = scan_i64_to_i64(w.longC, w.longCO, m, w.scan, w.scan_bytes, s);
         if (st != MSP_OK) return st;
+        }
     } else {
         st = cuda_check(cudaMemsetAsync(w.longpos, 0, sizeof(int64_t), s), "spgemm: clear");
         if (st == MSP_OK) st = cuda_check(cudaMemsetAsync(w.spapos, 0, sizeof(int64_t), s), "spgemm: clear");
