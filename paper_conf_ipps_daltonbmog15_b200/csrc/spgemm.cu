@@ -444,6 +444,9 @@ __global__ void wr_class_kernel(int32_t m, const int32_t *__restrict__ Arp, cons
 // C5 symbolic vs the loops' fraction of that), no global
 // scratch, no atomics outside shared memory.
 constexpr int WS_WARPS = 4;
+constexpr int WS_HASH_BITS = 9;  // symbolic: 512-slot (row, column) hash set per warp (load <= 1/2)
+constexpr int WS_HASH = 1 << WS_HASH_BITS;
+constexpr unsigned long long WS_EMPTY = ~0ull;
 template <typename V, bool NUM>
 __global__ void __launch_bounds__(WS_WARPS * 32, 8)
 ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const V *__restrict__ Aval,
@@ -453,22 +456,29 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const V *__restrict_
 {
     constexpr unsigned FULL = 0xffffffffu;
     __shared__ __align__(16) int32_t s_key_all[WS_WARPS][WS_BATCH];  // B: column by position
-    __shared__ int32_t s_b0_all[WS_WARPS][WS_BATCH];                 // A: B row start; D: head prefix H
-    __shared__ int16_t s_off_all[WS_WARPS][WS_BATCH + 2];            // A: product offset; D: sorted position | head
+    __shared__ int32_t s_b0_all[WS_WARPS][WS_BATCH];                 // A: B row start
+    __shared__ int16_t s_off_all[WS_WARPS][WS_BATCH + 2];            // A: product offset
+    __shared__ __align__(16) int16_t s_src_all[WS_WARPS][WS_BATCH];  // B: A nonzero (+1) of each position
     __shared__ unsigned s_first_all[NUM ? WS_WARPS : 1][WS_BATCH / 32];     // C: first-occurrence bits
-    __shared__ int s_cnt_all[WS_WARPS][32];                                   // C: symbolic row counts
+    __shared__ int s_cnt_all[WS_WARPS][32];                                   // C: symbolic duplicates per row
+    __shared__ unsigned long long s_hash_all[NUM ? 1 : WS_WARPS][NUM ? 1 : WS_HASH];  // C: symbolic (row, col) set
     __shared__ double s_val_all[NUM ? WS_WARPS : 1][NUM ? WS_BATCH : 1];
     __shared__ double s_av_all[NUM ? WS_WARPS : 1][NUM ? WS_BATCH : 1];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     int32_t *s_key = s_key_all[warp];
     int32_t *s_b0 = s_b0_all[warp];
     int16_t *s_off = s_off_all[warp];
+    int16_t *s_src = s_src_all[warp];
+    unsigned long long *s_hash = s_hash_all[NUM ? 0 : warp];
     unsigned *s_first = s_first_all[NUM ? warp : 0];
     int *s_cnt = s_cnt_all[warp];
     double *s_val = s_val_all[NUM ? warp : 0];
     double *s_av = s_av_all[NUM ? warp : 0];
     const int64_t nwarps = int64_t(gridDim.x) * WS_WARPS;
     s_cnt[lane] = 0;
+    reinterpret_cast<int4 *>(s_src)[lane] = make_int4(0, 0, 0, 0);
+    if constexpr (!NUM)
+        for (int i = lane; i < WS_HASH; i += 32) s_hash[i] = WS_EMPTY;
     for (int64_t r0 = (int64_t(blockIdx.x) * WS_WARPS + warp) * 32; r0 < m; r0 += nwarps * 32) {
         const int64_t r = r0 + lane;
         bool sm = false;
@@ -510,25 +520,42 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const V *__restrict_
                 if (i < na) {
                     const int32_t j = ja + i;
                     s_b0[i] = bstart[j];
-                    s_off[i] = int16_t(S[j] - base);
+                    const int64_t sj = S[j];
+                    const int off = int(sj - base);
+                    s_off[i] = int16_t(off);
+                    if (S[j + 1] > sj) s_src[off] = int16_t(i + 1);  // the A nonzero starting at this position
                     if constexpr (NUM) s_av[i] = double(Aval[j]);
                 }
             }
             __syncwarp();
             // ---- B: expand (all WS_PPL gathers of a lane in flight) ----
+            // every position's A nonzero: running max of the start marks
+            // (blocked, 8 positions per lane, then a warp max-scan)
+            {
+                const int4 w = reinterpret_cast<const int4 *>(s_src)[lane];
+                int v[8] = {w.x & 0xffff, int(uint32_t(w.x) >> 16), w.y & 0xffff, int(uint32_t(w.y) >> 16),
+                            w.z & 0xffff, int(uint32_t(w.z) >> 16), w.w & 0xffff, int(uint32_t(w.w) >> 16)};
+#pragma unroll
+                for (int q = 1; q < 8; ++q) v[q] = max(v[q], v[q - 1]);
+                int carry = v[7];
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const int t2 = __shfl_up_sync(FULL, carry, o);
+                    if (lane >= o) carry = max(carry, t2);
+                }
+                int prev = __shfl_up_sync(FULL, carry, 1);
+                if (lane == 0) prev = 0;
+#pragma unroll
+                for (int q = 0; q < 8; ++q) v[q] = max(v[q], prev);
+                reinterpret_cast<int4 *>(s_src)[lane] =
+                    make_int4(v[0] | (v[1] << 16), v[2] | (v[3] << 16), v[4] | (v[5] << 16), v[6] | (v[7] << 16));
+            }
+            __syncwarp();
             int pa[WS_PPL];  // A nonzero (batch index) of product u*32 + lane
 #pragma unroll
-            for (int u = 0; u < WS_PPL; ++u) pa[u] = 0;
-#pragma unroll
-            for (int stp = WS_BATCH / 2; stp >= 1; stp >>= 1) {
-                if (stp < na) {
-#pragma unroll
-                    for (int u = 0; u < WS_PPL; ++u) {
-                        const int c = pa[u] + stp;
-                        if (c < na && s_off[c] <= u * 32 + lane) pa[u] = c;
-                    }
-                }
-            }
+            for (int u = 0; u < WS_PPL; ++u) pa[u] = max(int(s_src[u * 32 + lane]) - 1, 0);
+            __syncwarp();
+            reinterpret_cast<int4 *>(s_src)[lane] = make_int4(0, 0, 0, 0);
             {
                 int32_t ck[WS_PPL];
                 double cv[WS_PPL];
@@ -569,9 +596,22 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const V *__restrict_
                 const bool act = p < np;
                 const int32_t c = act ? s_key[p] : 0;
                 if constexpr (!NUM) {
-                    bool first = act;
-                    for (int q = seg; q < p; ++q) first = first && (s_key[q] != c);
-                    if (first) atomicAdd(&s_cnt[t], 1);
+                    // distinct (row, column) pairs: insert into the warp's hash
+                    // set; an insert that finds its own key is a duplicate
+                    if (act) {
+                        const unsigned long long key = (static_cast<unsigned long long>(t) << 32) | uint32_t(c);
+                        uint32_t h = ((uint32_t(c) * 0x9E3779B1u) ^ (uint32_t(t) * 0x85EBCA77u)) >> (32 - WS_HASH_BITS);
+                        while (true) {
+                            const unsigned long long old = atomicCAS(&s_hash[h], WS_EMPTY, key);
+                            if (old == WS_EMPTY) break;
+                            if (old == key) {
+                                atomicAdd(&s_cnt[t], 1);
+                                break;
+                            }
+                            h = (h + 1) & (WS_HASH - 1);
+                        }
+                        s_off[p] = int16_t(h);  // (s_off is free after the expansion)
+                    }
                 } else {
                     const bool dupfree = __shfl_sync(FULL, U, t) == len;
                     if (act && dupfree) {
@@ -581,6 +621,12 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const V *__restrict_
                         Cval[rowc + rk] = V(s_val[p]);
                     }
                 }
+            }
+            if constexpr (!NUM) {
+                // clear the slots this batch used (a duplicate's probe ends on
+                // its first occurrence's slot: cleared twice, harmlessly)
+                __syncwarp();
+                for (int p = lane; p < np; p += 32) s_hash[s_off[p]] = WS_EMPTY;
             }
             if constexpr (NUM) {
                 // rows with duplicate columns: mark first occurrences, then rank
@@ -641,7 +687,7 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const V *__restrict_
         }
         if constexpr (!NUM) {
             __syncwarp();
-            if (sm) Crp[r + 1] = s_cnt[lane];  // Crp holds the row offsets: row r's count goes to Crp[r + 1]
+            if (sm) Crp[r + 1] = P - s_cnt[lane];  // Crp holds the row offsets: row r's count goes to Crp[r + 1]
             s_cnt[lane] = 0;
             __syncwarp();
         }
