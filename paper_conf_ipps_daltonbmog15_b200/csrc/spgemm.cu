@@ -415,82 +415,107 @@ __global__ void wr_class_kernel(int32_t m, const int32_t *__restrict__ Arp, cons
     }
 }
 
-// ------------------------------------------------ small rows (warp sort)
+// ------------------------------------------------ small rows
 // Rows with few products (C5's random rows: ~16; the uniform rows of C4) are
-// too small for a warp each and too wide for a bitmap.  A warp takes 32 rows
-// at a time (lane per row: mode, offsets) and processes runs of consecutive
-// SMALL rows with at most WS_BATCH products and A nonzeros together -- ESC
-// with the warp as the tile and the registers as the sort
-// buffer:
-//   A: lane per A nonzero j -- B row start (setup's bstart[j]) and product
-//      offset S[j] into shared memory (and a_ij, numeric);
-//   B: expansion, lane per product p (WS_PPL per lane, strided, all gathers
-//      in flight together): a search over the staged offsets finds p's A
-//      nonzero; the B column (and the fp64 product a_ik * b_kj, one rounding)
-//      lands at p in shared memory.  Positions follow Gustavson's order
-//      (k ascending, then B's order);
-//   C: compression, lane per product p of row r (segment [s_r, e_r) of the
-//      batch; rounds of 32 consecutive positions, each lane looping over its
-//      own row only).  p is the FIRST occurrence of its column c iff no q in
-//      [s_r, p) holds c; symbolic counts the first occurrences per row.
-//      Numeric: a row whose C row length equals P_r has no duplicates and
-//      p's rank is the number of smaller columns in the segment; otherwise
-//      first occurrences are marked (sign bit), each computes its rank among
-//      the marked columns and sums the products of c in position order
-//      (= k order: the oracle's order, separate roundings).  (c, sum) goes
-//      to C.rp[r] + rank.
-// O(P_r) work per product: fewer instructions than sorting the batch (a
-// 256-key bitonic network in registers measured 44 G warp instructions on
-// C5 symbolic vs the loops' fraction of that), no global
-// scratch, no atomics outside shared memory.
+// too small for a warp each and too wide for a bitmap.  ESC in
+// two passes per phase, so that the random B gathers and the per-row work
+// never wait on each other:
+//   expand (ws_expand_kernel): a thread per A nonzero j of a SMALL row
+//     copies its B row's columns (symbolic) or the fp64 products
+//     a_ik * b_kj, one rounding (numeric) to the product positions
+//     [S[j], S[j+1]) of a staging array in main_ws -- positions follow
+//     Gustavson's order (k ascending, then B's order); millions of
+//     independent threads keep the B-row gathers in flight (setup recorded
+//     each A nonzero's B row start, bstart[j], so no B offset is gathered);
+//   compress (ws_small_kernel): a warp takes 32 rows (lane per row: mode,
+//     offsets) and processes runs of consecutive SMALL rows with at most
+//     WS_BATCH products together: their staged products come in with
+//     coalesced loads (8 per lane in flight); then lane per product, rounds
+//     of 32 positions.  Symbolic: a shared-memory hash set of (row, column)
+//     counts each row's distinct columns (an insert that finds its own key is
+//     a duplicate).  Numeric: a row whose C length equals P_r has no
+//     duplicates and a product's rank is the number of smaller columns in its
+//     row; otherwise first occurrences (no equal column earlier in the row)
+//     are marked, each ranks among the marked columns and sums its column's
+//     products in position (= k) order -- the oracle's order, separate
+//     roundings -- and (c, sum) goes to C.rp[r] + rank.
+// O(P_r) work per product, cheap for small rows; no sort.
 constexpr int WS_WARPS = 4;
 constexpr int WS_HASH_BITS = 9;  // symbolic: 512-slot (row, column) hash set per warp (load <= 1/2)
 constexpr int WS_HASH = 1 << WS_HASH_BITS;
 constexpr unsigned long long WS_EMPTY = ~0ull;
+// expand: product position S[j] + q of A nonzero j (in a SMALL row) gets
+// B's column (symbolic) or the fp64 product a_ij * b_jq (numeric).
+template <typename V, bool NUM>
+__global__ void __launch_bounds__(256)
+ws_expand_kernel(int64_t nnzA, const int32_t *__restrict__ arow, const uint8_t *__restrict__ wmode,
+                 const int64_t *__restrict__ S, const int32_t *__restrict__ bstart, const V *__restrict__ Aval,
+                 const int32_t *__restrict__ Bcol, const V *__restrict__ Bval, int32_t *__restrict__ X,
+                 double *__restrict__ XV)
+{
+    const int64_t stride = int64_t(gridDim.x) * blockDim.x;
+    for (int64_t j = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; j < nnzA; j += stride) {
+        if (wmode[arow[j]] != WM_SMALL) continue;
+        const int64_t s0 = S[j];
+        const int len = int(S[j + 1] - s0);
+        const int32_t b0 = bstart[j];
+        if constexpr (!NUM) {
+            for (int q = 0; q < len; q += 4) {
+                int32_t c[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u) c[u] = (q + u < len) ? ldg64(Bcol + b0 + q + u) : 0;
+#pragma unroll
+                for (int u = 0; u < 4; ++u)
+                    if (q + u < len) X[s0 + q + u] = c[u];
+            }
+        } else {
+            const double a = double(Aval[j]);
+            for (int q = 0; q < len; q += 4) {
+                double v[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u) v[u] = (q + u < len) ? double(ldg64(Bval + b0 + q + u)) : 0.0;
+#pragma unroll
+                for (int u = 0; u < 4; ++u)
+                    if (q + u < len) XV[s0 + q + u] = __dmul_rn(a, v[u]);
+            }
+        }
+    }
+}
+
 template <typename V, bool NUM>
 __global__ void __launch_bounds__(WS_WARPS * 32, 8)
-ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const V *__restrict__ Aval,
-                const int32_t *__restrict__ bstart, const int32_t *__restrict__ Bcol, const V *__restrict__ Bval,
-                const uint8_t *__restrict__ wmode, const int64_t *__restrict__ S, int32_t *__restrict__ Crp,
-                int32_t *__restrict__ Ccol, V *__restrict__ Cval)
+ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__restrict__ wmode,
+                const int64_t *__restrict__ S, const int32_t *__restrict__ X, const double *__restrict__ XV,
+                int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol, V *__restrict__ Cval)
 {
     constexpr unsigned FULL = 0xffffffffu;
-    __shared__ __align__(16) int32_t s_key_all[WS_WARPS][WS_BATCH];  // B: column by position
-    __shared__ int32_t s_b0_all[WS_WARPS][WS_BATCH];                 // A: B row start
-    __shared__ int16_t s_off_all[WS_WARPS][WS_BATCH + 2];            // A: product offset
-    __shared__ __align__(16) int16_t s_src_all[WS_WARPS][WS_BATCH];  // B: A nonzero (+1) of each position
-    __shared__ unsigned s_first_all[NUM ? WS_WARPS : 1][WS_BATCH / 32];     // C: first-occurrence bits
-    __shared__ int s_cnt_all[WS_WARPS][32];                                   // C: symbolic duplicates per row
-    __shared__ unsigned long long s_hash_all[NUM ? 1 : WS_WARPS][NUM ? 1 : WS_HASH];  // C: symbolic (row, col) set
+    __shared__ __align__(16) int32_t s_key_all[WS_WARPS][WS_BATCH];  // column by batch position
+    __shared__ int16_t s_slot_all[NUM ? 1 : WS_WARPS][NUM ? 1 : WS_BATCH];  // symbolic: hash slot of each product
+    __shared__ unsigned s_first_all[NUM ? WS_WARPS : 1][WS_BATCH / 32];     // numeric: first-occurrence bits
+    __shared__ int s_cnt_all[WS_WARPS][32];                                   // symbolic: duplicates per row
+    __shared__ unsigned long long s_hash_all[NUM ? 1 : WS_WARPS][NUM ? 1 : WS_HASH];  // symbolic: (row, col) set
     __shared__ double s_val_all[NUM ? WS_WARPS : 1][NUM ? WS_BATCH : 1];
-    __shared__ double s_av_all[NUM ? WS_WARPS : 1][NUM ? WS_BATCH : 1];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     int32_t *s_key = s_key_all[warp];
-    int32_t *s_b0 = s_b0_all[warp];
-    int16_t *s_off = s_off_all[warp];
-    int16_t *s_src = s_src_all[warp];
+    int16_t *s_slot = s_slot_all[NUM ? 0 : warp];
     unsigned long long *s_hash = s_hash_all[NUM ? 0 : warp];
     unsigned *s_first = s_first_all[NUM ? warp : 0];
     int *s_cnt = s_cnt_all[warp];
     double *s_val = s_val_all[NUM ? warp : 0];
-    double *s_av = s_av_all[NUM ? warp : 0];
     const int64_t nwarps = int64_t(gridDim.x) * WS_WARPS;
     s_cnt[lane] = 0;
-    reinterpret_cast<int4 *>(s_src)[lane] = make_int4(0, 0, 0, 0);
     if constexpr (!NUM)
         for (int i = lane; i < WS_HASH; i += 32) s_hash[i] = WS_EMPTY;
     for (int64_t r0 = (int64_t(blockIdx.x) * WS_WARPS + warp) * 32; r0 < m; r0 += nwarps * 32) {
         const int64_t r = r0 + lane;
         bool sm = false;
-        int32_t a0 = 0, a1 = 0, cb = 0;
+        int32_t cb = 0;
         int64_t p0 = 0;
         int P = 0, U = 0;
         if (r < m && wmode[r] == WM_SMALL) {
             sm = true;
-            a0 = Arp[r];
-            a1 = Arp[r + 1];
-            p0 = S[a0];
-            P = int(S[a1] - p0);
+            p0 = S[Arp[r]];
+            P = int(S[Arp[r + 1]] - p0);
             if (NUM) {
                 cb = Crp[r];
                 U = Crp[r + 1] - cb;  // == P: no duplicate columns in the row
@@ -498,77 +523,26 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const V *__restrict_
         }
         unsigned todo = __ballot_sync(FULL, sm);
         while (todo) {
-            // batch: the run of consecutive SMALL lanes from s whose products
-            // and A nonzeros fit
+            // batch: the run of consecutive SMALL lanes from s whose products fit
             const int s = __ffs(todo) - 1;
             const int64_t base = __shfl_sync(FULL, p0, s);
-            const int32_t ja = __shfl_sync(FULL, a0, s);
-            const bool fits = sm && lane >= s && (p0 + P - base) <= WS_BATCH && a1 - ja <= WS_BATCH;
+            const bool fits = sm && lane >= s && (p0 + P - base) <= WS_BATCH;
             const unsigned fm = __ballot_sync(FULL, fits) >> s;
             const int run = (~fm) ? __ffs(~fm) - 1 : 32 - s;
             const int e = s + run;  // lanes [s, e)
             todo &= ~unsigned(((1ull << run) - 1ull) << s);
-            const int32_t jb = __shfl_sync(FULL, a1, e - 1);
-            const int na = jb - ja;
             const int np = int(__shfl_sync(FULL, p0, e - 1) - base) + __shfl_sync(FULL, P, e - 1);
             const int prel = int(p0 - base);  // this lane's row start in the batch (lanes in [s, e))
             const bool inb = lane >= s && lane < e;
-            // ---- A: stage the batch's A nonzeros ----
-#pragma unroll
-            for (int u = 0; u < WS_PPL; ++u) {
-                const int i = u * 32 + lane;
-                if (i < na) {
-                    const int32_t j = ja + i;
-                    s_b0[i] = bstart[j];
-                    const int64_t sj = S[j];
-                    const int off = int(sj - base);
-                    s_off[i] = int16_t(off);
-                    if (S[j + 1] > sj) s_src[off] = int16_t(i + 1);  // the A nonzero starting at this position
-                    if constexpr (NUM) s_av[i] = double(Aval[j]);
-                }
-            }
-            __syncwarp();
-            // ---- B: expand (all WS_PPL gathers of a lane in flight) ----
-            // every position's A nonzero: running max of the start marks
-            // (blocked, 8 positions per lane, then a warp max-scan)
-            {
-                const int4 w = reinterpret_cast<const int4 *>(s_src)[lane];
-                int v[8] = {w.x & 0xffff, int(uint32_t(w.x) >> 16), w.y & 0xffff, int(uint32_t(w.y) >> 16),
-                            w.z & 0xffff, int(uint32_t(w.z) >> 16), w.w & 0xffff, int(uint32_t(w.w) >> 16)};
-#pragma unroll
-                for (int q = 1; q < 8; ++q) v[q] = max(v[q], v[q - 1]);
-                int carry = v[7];
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const int t2 = __shfl_up_sync(FULL, carry, o);
-                    if (lane >= o) carry = max(carry, t2);
-                }
-                int prev = __shfl_up_sync(FULL, carry, 1);
-                if (lane == 0) prev = 0;
-#pragma unroll
-                for (int q = 0; q < 8; ++q) v[q] = max(v[q], prev);
-                reinterpret_cast<int4 *>(s_src)[lane] =
-                    make_int4(v[0] | (v[1] << 16), v[2] | (v[3] << 16), v[4] | (v[5] << 16), v[6] | (v[7] << 16));
-            }
-            __syncwarp();
-            int pa[WS_PPL];  // A nonzero (batch index) of product u*32 + lane
-#pragma unroll
-            for (int u = 0; u < WS_PPL; ++u) pa[u] = max(int(s_src[u * 32 + lane]) - 1, 0);
-            __syncwarp();
-            reinterpret_cast<int4 *>(s_src)[lane] = make_int4(0, 0, 0, 0);
+            // ---- the batch's staged products: coalesced, all loads in flight ----
             {
                 int32_t ck[WS_PPL];
                 double cv[WS_PPL];
 #pragma unroll
                 for (int u = 0; u < WS_PPL; ++u) {
                     const int p = u * 32 + lane;
-                    ck[u] = 0;
-                    cv[u] = 0.0;
-                    if (p < np) {
-                        const int32_t bi = s_b0[pa[u]] + (p - s_off[pa[u]]);
-                        ck[u] = ldg64(Bcol + bi);
-                        if constexpr (NUM) cv[u] = __dmul_rn(s_av[pa[u]], double(ldg64(Bval + bi)));
-                    }
+                    ck[u] = p < np ? X[base + p] : 0;
+                    if constexpr (NUM) cv[u] = p < np ? XV[base + p] : 0.0;
                 }
 #pragma unroll
                 for (int u = 0; u < WS_PPL; ++u) {
@@ -610,7 +584,7 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const V *__restrict_
                             }
                             h = (h + 1) & (WS_HASH - 1);
                         }
-                        s_off[p] = int16_t(h);  // (s_off is free after the expansion)
+                        s_slot[p] = int16_t(h);
                     }
                 } else {
                     const bool dupfree = __shfl_sync(FULL, U, t) == len;
@@ -626,7 +600,7 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const V *__restrict_
                 // clear the slots this batch used (a duplicate's probe ends on
                 // its first occurrence's slot: cleared twice, harmlessly)
                 __syncwarp();
-                for (int p = lane; p < np; p += 32) s_hash[s_off[p]] = WS_EMPTY;
+                for (int p = lane; p < np; p += 32) s_hash[s_slot[p]] = WS_EMPTY;
             }
             if constexpr (NUM) {
                 // rows with duplicate columns: mark first occurrences, then rank
@@ -1633,6 +1607,8 @@ struct MainWs {
     GSplit *splits;
     uint16_t *perm;  // per tile: the symbolic sort's permutation (GM_T entries)
     int32_t *ucol;   // row-accumulator path: each short row's output columns at its product offset
+    int32_t *xcol;   // small-row path: B column of every product (symbolic expand; numeric reads it)
+    double *xval;    // small-row path: every product a_ik * b_kj (numeric expand)
     int32_t *Xc[2];
     double *Xv[2];
     int32_t *heads;
@@ -1643,13 +1619,15 @@ struct MainWs {
     size_t bytes;
 };
 
-MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, int64_t nucol, void *ws, size_t cap, bool *ok)
+MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, int64_t nucol, int64_t nx, void *ws, size_t cap, bool *ok)
 {
     MainWs w;
     Carve cv(ws, cap);
     w.splits = cv.take<GSplit>(size_t(ntiles + 1));
     w.perm = cv.take<uint16_t>(size_t(ntiles) * GM_T);
     w.ucol = cv.take<int32_t>(size_t(nucol > 0 ? nucol : 1));
+    w.xcol = cv.take<int32_t>(size_t(nx > 0 ? nx : 1));
+    w.xval = cv.take<double>(size_t(nx > 0 ? nx : 1));
     for (int i = 0; i < 2; ++i) {
         w.Xc[i] = cv.take<int32_t>(size_t(LP > 0 ? LP : 1));
         w.Xv[i] = cv.take<double>(size_t(LP > 0 ? LP : 1));
@@ -1823,19 +1801,23 @@ bool small_enabled()
 }
 
 template <typename V, bool NUM>
-msp_status run_small(const msp_csr *A, const msp_csr *B, const SetupWs &sw, int32_t *Crp, int32_t *Ccol, void *Cval,
-                     cudaStream_t s)
+msp_status run_small(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, int32_t *Crp,
+                     int32_t *Ccol, void *Cval, cudaStream_t s)
 {
+    const int64_t nnz = A->nnz;
+    ws_expand_kernel<V, NUM><<<unsigned(std::min<int64_t>(ceil_div(nnz, 256), 148 * 32)), 256, 0, s>>>(
+        nnz, sw.arow, sw.wmode, sw.S, sw.bstart, static_cast<const V *>(A->vals), B->col_idx,
+        static_cast<const V *>(B->vals), mw.xcol, mw.xval);
+    msp_status st = last_launch(NUM ? "ws_expand_kernel<numeric>" : "ws_expand_kernel<symbolic>");
+    if (st != MSP_OK) return st;
     auto kern = ws_small_kernel<V, NUM>;
     int occ = 1;
-    msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), 0, "spgemm: small rows", WS_WARPS * 32, &occ,
-                                  true);
+    st = set_smem_attr(reinterpret_cast<const void *>(kern), 0, "spgemm: small rows", WS_WARPS * 32, &occ, true);
     if (st != MSP_OK) return st;
     const int32_t m = A->nrows;
     const int64_t g = std::min<int64_t>(int64_t(occ) * sm_count(), ceil_div(m, WS_WARPS * 32));
-    kern<<<unsigned(g > 0 ? g : 1), WS_WARPS * 32, 0, s>>>(m, A->row_offsets, static_cast<const V *>(A->vals),
-                                                          sw.bstart, B->col_idx, static_cast<const V *>(B->vals),
-                                                          sw.wmode, sw.S, Crp, Ccol, static_cast<V *>(Cval));
+    kern<<<unsigned(g > 0 ? g : 1), WS_WARPS * 32, 0, s>>>(m, A->row_offsets, sw.wmode, sw.S, mw.xcol, mw.xval, Crp,
+                                                          Ccol, static_cast<V *>(Cval));
     return last_launch(NUM ? "ws_small_kernel<numeric>" : "ws_small_kernel<symbolic>");
 }
 
@@ -1845,8 +1827,8 @@ msp_status run_rowacc(const msp_csr *A, const msp_csr *B, const SetupWs &sw, con
 {
     const int32_t m = A->nrows;
     if (h.nsmall > 0) {
-        msp_status st = (A->dtype == MSP_F64) ? run_small<double, NUM>(A, B, sw, Crp, Ccol, Cval, s)
-                                              : run_small<float, NUM>(A, B, sw, Crp, Ccol, Cval, s);
+        msp_status st = (A->dtype == MSP_F64) ? run_small<double, NUM>(A, B, sw, mw, Crp, Ccol, Cval, s)
+                                              : run_small<float, NUM>(A, B, sw, mw, Crp, Ccol, Cval, s);
         if (st != MSP_OK) return st;
     }
     if (h.nbitmap <= 0) return MSP_OK;
@@ -1936,8 +1918,8 @@ msp_status prepare_main(const msp_csr *A, const void *ws1, size_t b1, void *ws2,
     bool ok1, ok2;
     *sw = carve_setup(A, const_cast<void *>(ws1), b1, &ok1);
     if (!ok1) return MSP_ERR_WORKSPACE;
-    *mw = carve_main(A->nrows, ntiles_of(A->nnz, h.nprods, h.rowacc), h.LP, h.nbitmap > 0 ? h.nprods : 0, ws2, b2,
-                     &ok2);
+    *mw = carve_main(A->nrows, ntiles_of(A->nnz, h.nprods, h.rowacc), h.LP, h.nbitmap > 0 ? h.nprods : 0,
+                     h.nsmall > 0 ? h.nprods : 0, ws2, b2, &ok2);
     if (!ok2) return MSP_ERR_WORKSPACE;
     return MSP_OK;
 }
@@ -2064,7 +2046,8 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
     if (st != MSP_OK) return st;
     const int64_t ntiles = ntiles_of(nnz, h.nprods, h.rowacc);
     bool ok2;
-    MainWs mw = carve_main(m, ntiles, h.LP, h.nbitmap > 0 ? h.nprods : 0, nullptr, SIZE_MAX, &ok2);
+    MainWs mw = carve_main(m, ntiles, h.LP, h.nbitmap > 0 ? h.nprods : 0, h.nsmall > 0 ? h.nprods : 0, nullptr,
+                           SIZE_MAX, &ok2);
     info->nprods = h.nprods;
     info->ntiles = ntiles;
     info->long_rows = h.nlong;
