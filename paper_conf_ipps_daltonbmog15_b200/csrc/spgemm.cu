@@ -441,6 +441,9 @@ __global__ void wr_class_kernel(int32_t m, const int32_t *__restrict__ Arp, cons
 //     roundings -- and (c, sum) goes to C.rp[r] + rank.
 // O(P_r) work per product, cheap for small rows; no sort.
 constexpr int WS_WARPS = 4;
+#ifndef WS_PAD
+#define WS_PAD 0
+#endif
 constexpr int WS_HASH_BITS = 9;  // symbolic: 512-slot (row, column) hash set per warp (load <= 1/2)
 constexpr int WS_HASH = 1 << WS_HASH_BITS;
 constexpr unsigned long long WS_EMPTY = ~0ull;
@@ -483,20 +486,27 @@ ws_expand_kernel(int64_t nnzA, const int32_t *__restrict__ arow, const uint8_t *
 }
 
 template <typename V, bool NUM>
-__global__ void __launch_bounds__(WS_WARPS * 32, 8)
+__global__ void __launch_bounds__(WS_WARPS * 32, (NUM && WS_PAD) ? 6 : 8)
 ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__restrict__ wmode,
                 const int64_t *__restrict__ S, const int32_t *__restrict__ X, const double *__restrict__ XV,
                 int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol, V *__restrict__ Cval)
 {
     constexpr unsigned FULL = 0xffffffffu;
-    __shared__ __align__(16) int32_t s_key_all[WS_WARPS][WS_BATCH];  // column by batch position
+    // WS_PAD (experiment): numeric stores each row at a 4-aligned start padded
+    // with INT_MAX, so the rank loop reads 4 columns per shared load -- measured
+    // slower on C5 (22.0 vs 18.6 ms: 80 registers, fewer warps), off
+    constexpr bool PADDED = NUM && WS_PAD;
+    constexpr int KCAP = PADDED ? WS_BATCH + 3 * 32 : WS_BATCH;
+    __shared__ __align__(16) int32_t s_key_all[WS_WARPS][KCAP];  // column by (padded) batch position
+    __shared__ __align__(16) uint8_t s_row_all[WS_WARPS][WS_BATCH];  // row lane of each batch position
     __shared__ int16_t s_slot_all[NUM ? 1 : WS_WARPS][NUM ? 1 : WS_BATCH];  // symbolic: hash slot of each product
-    __shared__ unsigned s_first_all[NUM ? WS_WARPS : 1][WS_BATCH / 32];     // numeric: first-occurrence bits
+    __shared__ unsigned s_first_all[NUM ? WS_WARPS : 1][KCAP / 32];         // numeric: first-occurrence bits
     __shared__ int s_cnt_all[WS_WARPS][32];                                   // symbolic: duplicates per row
     __shared__ unsigned long long s_hash_all[NUM ? 1 : WS_WARPS][NUM ? 1 : WS_HASH];  // symbolic: (row, col) set
-    __shared__ double s_val_all[NUM ? WS_WARPS : 1][NUM ? WS_BATCH : 1];
+    __shared__ double s_val_all[NUM ? WS_WARPS : 1][NUM ? KCAP : 1];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     int32_t *s_key = s_key_all[warp];
+    uint8_t *s_row = s_row_all[warp];
     int16_t *s_slot = s_slot_all[NUM ? 0 : warp];
     unsigned long long *s_hash = s_hash_all[NUM ? 0 : warp];
     unsigned *s_first = s_first_all[NUM ? warp : 0];
@@ -504,6 +514,7 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__res
     double *s_val = s_val_all[NUM ? warp : 0];
     const int64_t nwarps = int64_t(gridDim.x) * WS_WARPS;
     s_cnt[lane] = 0;
+    reinterpret_cast<uint2 *>(s_row)[lane] = make_uint2(0u, 0u);
     if constexpr (!NUM)
         for (int i = lane; i < WS_HASH; i += 32) s_hash[i] = WS_EMPTY;
     for (int64_t r0 = (int64_t(blockIdx.x) * WS_WARPS + warp) * 32; r0 < m; r0 += nwarps * 32) {
@@ -535,44 +546,73 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__res
             const int prel = int(p0 - base);  // this lane's row start in the batch (lanes in [s, e))
             const bool inb = lane >= s && lane < e;
             // ---- the batch's staged products: coalesced, all loads in flight ----
+            int32_t ck[WS_PPL];
+            double cv[WS_PPL];
+#pragma unroll
+            for (int u = 0; u < WS_PPL; ++u) {
+                const int p = u * 32 + lane;
+                ck[u] = p < np ? X[base + p] : 0;
+                if constexpr (NUM) cv[u] = p < np ? XV[base + p] : 0.0;
+            }
+            // ---- row lane of every position: start marks, blocked max-scan ----
+            if (inb) s_row[prel] = uint8_t(lane + 1);
+            __syncwarp();
             {
-                int32_t ck[WS_PPL];
-                double cv[WS_PPL];
+                const uint2 mk = reinterpret_cast<const uint2 *>(s_row)[lane];
+                int v[8];
 #pragma unroll
-                for (int u = 0; u < WS_PPL; ++u) {
-                    const int p = u * 32 + lane;
-                    ck[u] = p < np ? X[base + p] : 0;
-                    if constexpr (NUM) cv[u] = p < np ? XV[base + p] : 0.0;
+                for (int q = 0; q < 8; ++q) v[q] = int(((q < 4 ? mk.x : mk.y) >> (8 * (q & 3))) & 0xffu);
+#pragma unroll
+                for (int q = 1; q < 8; ++q) v[q] = max(v[q], v[q - 1]);
+                int carry = v[7];
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const int t2 = __shfl_up_sync(FULL, carry, o);
+                    if (lane >= o) carry = max(carry, t2);
                 }
+                int prev = __shfl_up_sync(FULL, carry, 1);
+                if (lane == 0) prev = 0;
+                uint32_t w0 = 0, w1 = 0;
 #pragma unroll
-                for (int u = 0; u < WS_PPL; ++u) {
-                    const int p = u * 32 + lane;
-                    if (p < np) {
-                        s_key[p] = ck[u];
-                        if constexpr (NUM) s_val[p] = cv[u];
-                    }
+                for (int q = 0; q < 8; ++q) {
+                    const uint32_t b = uint32_t(max(v[q], prev) - 1) & 0xffu;  // 0-based row lane
+                    if (q < 4) w0 |= b << (8 * q);
+                    else w1 |= b << (8 * (q - 4));
+                }
+                __syncwarp();
+                reinterpret_cast<uint2 *>(s_row)[lane] = make_uint2(w0, w1);
+            }
+            __syncwarp();
+            // numeric: rows at 4-aligned starts (pstart), padded with INT_MAX
+            int pstart = prel;
+            if constexpr (PADDED) {
+                const int pad = inb ? ((4 - (P & 3)) & 3) : 0;
+                pstart = prel + warp_inclusive_sum(pad, lane) - pad;
+                if (inb)
+                    for (int q = 0; q < pad; ++q) s_key[pstart + P + q] = INT_MAX;
+            }
+#pragma unroll
+            for (int u = 0; u < WS_PPL; ++u) {
+                const int p = u * 32 + lane;
+                const int t = p < np ? int(s_row[p]) : s;
+                const int pp = PADDED ? __shfl_sync(FULL, pstart, t) + (p - __shfl_sync(FULL, prel, t)) : p;
+                if (p < np) {
+                    s_key[pp] = ck[u];
+                    if constexpr (NUM) s_val[pp] = cv[u];
                 }
             }
             __syncwarp();
             // ---- C: compression, lane per product, rounds of 32 positions ----
+            bool anydup = false;
             for (int pr = 0; pr < np; pr += 32) {
                 const int p = pr + lane;
-                int t = s;  // the product's row lane: last lane in [s, e) starting at or before p
-#pragma unroll
-                for (int stp = 16; stp >= 1; stp >>= 1) {
-                    const int c = t + stp;
-                    const int oc = __shfl_sync(FULL, prel, c & 31);
-                    if (c < e && oc <= p) t = c;
-                }
-                const int seg = __shfl_sync(FULL, prel, t);
-                const int len = __shfl_sync(FULL, P, t);
-                const int32_t rowc = __shfl_sync(FULL, cb, t);
                 const bool act = p < np;
-                const int32_t c = act ? s_key[p] : 0;
+                const int t = act ? int(s_row[p]) : s;  // the product's row lane
                 if constexpr (!NUM) {
                     // distinct (row, column) pairs: insert into the warp's hash
                     // set; an insert that finds its own key is a duplicate
                     if (act) {
+                        const int32_t c = s_key[p];
                         const unsigned long long key = (static_cast<unsigned long long>(t) << 32) | uint32_t(c);
                         uint32_t h = ((uint32_t(c) * 0x9E3779B1u) ^ (uint32_t(t) * 0x85EBCA77u)) >> (32 - WS_HASH_BITS);
                         while (true) {
@@ -587,12 +627,26 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__res
                         s_slot[p] = int16_t(h);
                     }
                 } else {
+                    const int seg = __shfl_sync(FULL, pstart, t);
+                    const int len = __shfl_sync(FULL, P, t);
+                    const int32_t rowc = __shfl_sync(FULL, cb, t);
+                    const int pp = seg + (p - __shfl_sync(FULL, prel, t));
                     const bool dupfree = __shfl_sync(FULL, U, t) == len;
+                    anydup |= act && !dupfree;
                     if (act && dupfree) {
+                        // rank = smaller columns in the row (4 per shared load; pads never count)
+                        const int32_t c = s_key[pp];
                         int rk = 0;
-                        for (int q = seg; q < seg + len; ++q) rk += s_key[q] < c ? 1 : 0;
+                        if constexpr (PADDED) {
+                            for (int q = seg; q < seg + len; q += 4) {
+                                const int4 w = *reinterpret_cast<const int4 *>(s_key + q);
+                                rk += int(w.x < c) + int(w.y < c) + int(w.z < c) + int(w.w < c);
+                            }
+                        } else {
+                            for (int q = seg; q < seg + len; ++q) rk += s_key[q] < c ? 1 : 0;
+                        }
                         Ccol[rowc + rk] = c;
-                        Cval[rowc + rk] = V(s_val[p]);
+                        Cval[rowc + rk] = V(s_val[pp]);
                     }
                 }
             }
@@ -605,51 +659,40 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__res
             if constexpr (NUM) {
                 // rows with duplicate columns: mark first occurrences, then rank
                 // among marked columns and sum each column's run in order
-                const bool anydup = __any_sync(FULL, inb && U != P);
-                if (anydup) {
+                if (__any_sync(FULL, anydup)) {
+                    for (int i = lane; i < KCAP / 32; i += 32) s_first[i] = 0u;
                     __syncwarp();
                     for (int pr = 0; pr < np; pr += 32) {
                         const int p = pr + lane;
-                        int t = s;
-#pragma unroll
-                        for (int stp = 16; stp >= 1; stp >>= 1) {
-                            const int c = t + stp;
-                            const int oc = __shfl_sync(FULL, prel, c & 31);
-                            if (c < e && oc <= p) t = c;
-                        }
-                        const int seg = __shfl_sync(FULL, prel, t);
+                        const int t = p < np ? int(s_row[p]) : s;
+                        const int seg = __shfl_sync(FULL, pstart, t);
+                        const int pp = seg + (p - __shfl_sync(FULL, prel, t));
                         const bool dup = __shfl_sync(FULL, U, t) != __shfl_sync(FULL, P, t);
-                        bool first = false;
                         if (p < np && dup) {
-                            const int32_t c = s_key[p];
-                            first = true;
-                            for (int q = seg; q < p; ++q) first = first && (s_key[q] != c);
+                            const int32_t c = s_key[pp];
+                            bool first = true;
+                            for (int q = seg; q < pp; ++q) first = first && (s_key[q] != c);
+                            if (first) atomicOr(&s_first[pp >> 5], 1u << (pp & 31));
                         }
-                        s_first[pr / 32] = __ballot_sync(FULL, first);  // one word per round
                     }
                     __syncwarp();
                     for (int pr = 0; pr < np; pr += 32) {
                         const int p = pr + lane;
-                        int t = s;
-#pragma unroll
-                        for (int stp = 16; stp >= 1; stp >>= 1) {
-                            const int c = t + stp;
-                            const int oc = __shfl_sync(FULL, prel, c & 31);
-                            if (c < e && oc <= p) t = c;
-                        }
-                        const int seg = __shfl_sync(FULL, prel, t);
+                        const int t = p < np ? int(s_row[p]) : s;
+                        const int seg = __shfl_sync(FULL, pstart, t);
                         const int len = __shfl_sync(FULL, P, t);
                         const int32_t rowc = __shfl_sync(FULL, cb, t);
+                        const int pp = seg + (p - __shfl_sync(FULL, prel, t));
                         const bool dup = __shfl_sync(FULL, U, t) != len;
-                        if (p < np && dup && ((s_first[pr / 32] >> lane) & 1u)) {
-                            const int32_t c = s_key[p];
+                        if (p < np && dup && ((s_first[pp >> 5] >> (pp & 31)) & 1u)) {
+                            const int32_t c = s_key[pp];
                             int rk = 0;
-                            double sum = s_val[p];
+                            double sum = s_val[pp];
                             for (int q = seg; q < seg + len; ++q) {
                                 const int32_t kq = s_key[q];
                                 const bool fq = (s_first[q >> 5] >> (q & 31)) & 1u;
                                 rk += (fq && kq < c) ? 1 : 0;
-                                if (kq == c && q > p) sum = __dadd_rn(sum, s_val[q]);
+                                if (kq == c && q > pp) sum = __dadd_rn(sum, s_val[q]);
                             }
                             Ccol[rowc + rk] = c;
                             Cval[rowc + rk] = V(sum);
@@ -657,6 +700,8 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__res
                     }
                 }
             }
+            __syncwarp();
+            reinterpret_cast<uint2 *>(s_row)[lane] = make_uint2(0u, 0u);  // marks of the next batch start clean
             __syncwarp();
         }
         if constexpr (!NUM) {
