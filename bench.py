@@ -136,11 +136,14 @@ def spgemm_pass_bytes(m, nnz_a, nprods, nnz_c, vsize, rowacc=False, small=False)
     """The method's own traffic per pass.  Small-row path
     (small, every short row has few products): setup as below plus the B row
     start of every A nonzero (4) and the row classification (A offsets and 16
-    of S per row); symbolic reads each A nonzero's B row start and S (12),
-    gathers one B column per product (4), reads A offsets and S per row (24)
-    and writes C's row counts (4 per row); numeric reads the same plus A
-    values (12 + s per A nonzero), C's row offsets (8 per row), gathers a B
-    column + value per product (4 + s) and writes C (4 + s per C nonzero).
+    of S per row).  Symbolic = expand (per A nonzero: COO row, B row start,
+    S[j], S[j+1], row mode: 4 + 4 + 16 + 1; per product: one B column
+    gathered (4) and staged (4)) + compress (per product: the staged column
+    (4); per row: mode, A offsets, S, the count written: 1 + 8 + 16 + 4).
+    Numeric = expand (the same per A nonzero plus a_ij (s); per product a B
+    value gathered (s) and the fp64 product staged (8)) + compress (per
+    product: staged product (8) and column (4) read; per row: mode, A
+    offsets, S, C offsets; C written (4 + s per C nonzero)).
     Row accumulator (rowacc): setup as below plus the span pass (A columns,
     8 of B offsets and 8 of B columns per A nonzero); symbolic reads A columns and B offsets
     (12 per A nonzero), gathers one B column per product (4) and writes each
@@ -158,9 +161,13 @@ def spgemm_pass_bytes(m, nnz_a, nprods, nnz_c, vsize, rowacc=False, small=False)
                 permutation read (2), C columns + values written (4 + s)."""
     setup = 4 * (m + 1) + nnz_a * (4 + 8 + 8 + 4)
     if small:
+        # expand + compress: the expand pass writes each product's column
+        # (symbolic, 4) or fp64 product (numeric, 8) to a staging array that
+        # the compress pass reads back (numeric also reads the columns)
         setup += nnz_a * 4 + m * (8 + 16)
-        symbolic = nnz_a * 12 + nprods * 4 + m * (24 + 4)
-        numeric = nnz_a * (12 + vsize) + nprods * (4 + vsize) + nnz_c * (4 + vsize) + m * (24 + 8)
+        symbolic = nnz_a * (4 + 4 + 16 + 1) + nprods * (4 + 4 + 4) + m * (1 + 8 + 16 + 4)
+        numeric = (nnz_a * (4 + 4 + 16 + 1 + vsize) + nprods * (vsize + 8 + 8 + 4) + nnz_c * (4 + vsize)
+                   + m * (1 + 8 + 16 + 8))
         return {"setup": setup, "symbolic": symbolic, "numeric": numeric}
     if rowacc:
         setup += 4 * (m + 1) + nnz_a * (4 + 8 + 8)
