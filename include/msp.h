@@ -211,11 +211,15 @@ typedef struct {
     int64_t long_chunks;     /* sorted chunks of the long-row pass */
     int64_t max_tile_span;   /* largest row span of a product tile: -1 after
                                 setup, set by symbolic (picks the key width) */
-    int64_t segmented_rows;  /* long rows taking the segmented (row-wise dense
-                                accumulator) path instead of the ESC long-row
-                                pass: output span <= 12288 columns and >= 1
-                                product per 4 columns of it (
-                                MSP_SPGEMM_SEGMENTED=0 disables) */
+    int64_t segmented_rows;  /* windows (CTAs) of the long rows taking the
+                                segmented (dense accumulator) path instead of
+                                the ESC long-row pass: >= 1 product per 4
+                                columns of the output span; a span wider than
+                                12,288 columns is cut into 12,288-column
+                                windows while windows x nnz(A row) <=
+                                products (one window per row otherwise, so
+                                for narrow rows this counts rows; SURVEY §8(f)
+                                f3; MSP_SPGEMM_SEGMENTED=0 disables) */
     int64_t row_accumulator; /* > 0: every short row's output span is at most
                                 65,536 columns (the value is the widest
                                 span, which sizes the bitmaps), so the short

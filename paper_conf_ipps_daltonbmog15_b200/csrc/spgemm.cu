@@ -180,7 +180,14 @@ __global__ void span_kernel(int64_t nnzA, const int32_t *__restrict__ Acol, cons
     }
 }
 
-// cost model: segmented iff span <= SPA_W and P_r >= span / 4
+// Cost model: a long row is segmented iff its products cover at least one
+// column in four of its output span (P_r >= span / 4).  A span wider than
+// SPA_W is cut into windows of SPA_W columns, one CTA each (every window CTA
+// walks all of the row's A nonzeros and binary-searches each B row for its
+// window), taken only while those searches stay below the product work:
+// windows * nnz_r <= P_r (C4's rows through the dense row: 163 windows x ~10
+// A nonzeros for 4.75e6 products; the dense row itself, 10^6 A nonzeros,
+// stays on the ESC long-row pass).  spaflag[r] = the row's window count.
 __global__ void spa_classify_kernel(int32_t m, const int32_t *__restrict__ rp, const int64_t *__restrict__ S,
                                     const int32_t *__restrict__ lo, const int32_t *__restrict__ hi,
                                     uint8_t *__restrict__ rowlong, int32_t *__restrict__ longflag,
@@ -191,8 +198,9 @@ __global__ void spa_classify_kernel(int32_t m, const int32_t *__restrict__ rp, c
         if (rowlong[r]) {
             const int64_t span = int64_t(hi[r]) - lo[r] + 1;
             const int64_t P = S[rp[r + 1]] - S[rp[r]];
-            if (span >= 1 && span <= SPA_W && 4 * P >= span) {
-                f = 1;
+            const int64_t nwin = (span + SPA_W - 1) / SPA_W;
+            if (span >= 1 && 4 * P >= span && (nwin == 1 || nwin * int64_t(rp[r + 1] - rp[r]) <= P)) {
+                f = int(nwin);
                 rowlong[r] = 2;   // masked in tiles like a long row
                 longflag[r] = 0;  // not in the ESC long-row pass
             }
@@ -201,40 +209,82 @@ __global__ void spa_classify_kernel(int32_t m, const int32_t *__restrict__ rp, c
     }
 }
 
-__global__ void spa_scatter_kernel(int32_t m, const int32_t *__restrict__ spaflag, const int64_t *__restrict__ spapos,
-                                   int32_t *__restrict__ sparow)
-{
-    for (int64_t r = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; r < m; r += int64_t(gridDim.x) * blockDim.x)
-        if (spaflag[r]) sparow[spapos[r]] = int32_t(r);
-}
+// The segmented rows' windows are numbered in row order by the exclusive
+// scan spapos of spaflag: item i belongs to the row r with spapos[r] <= i <
+// spapos[r+1] and is its window i - spapos[r].
 
-// One CTA per segmented row.  Symbolic marks the row's output columns (no
-// ordering needed) and counts them; numeric accumulates a_ik * b_kj for k in
-// A's column order (a barrier per A nonzero keeps every column's sum in that
-// order), then writes the marked columns ascending at C.rp[r].
+// One CTA per window of a segmented row (rows with span <= SPA_W: one
+// window).  Symbolic marks the window's output columns (no ordering needed),
+// counts them into C.rp[r+1] (atomic: integers, order-free) and keeps the
+// window's count in wcnt[item]; numeric accumulates a_ik * b_kj for k in A's
+// column order (a barrier per A nonzero keeps every column's sum in that
+// order), then writes the marked columns ascending at C.rp[r] + the counts
+// of the row's earlier windows.
 template <typename V, bool NUM>
 __global__ void __launch_bounds__(SPA_NT)
-spa_row_kernel(const int32_t *__restrict__ sparow, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
-               const V *__restrict__ Aval, const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
-               const V *__restrict__ Bval, const int32_t *__restrict__ spanlo, const int32_t *__restrict__ spanhi,
-               int32_t *__restrict__ Crp_counts, const int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol,
-               V *__restrict__ Cval)
+spa_row_kernel(int32_t m, const int64_t *__restrict__ spapos, const int32_t *__restrict__ Arp,
+               const int32_t *__restrict__ Acol, const V *__restrict__ Aval, const int32_t *__restrict__ Brp,
+               const int32_t *__restrict__ Bcol, const V *__restrict__ Bval, const int32_t *__restrict__ spanlo,
+               const int32_t *__restrict__ spanhi, int32_t *__restrict__ Crp_counts, const int32_t *__restrict__ Crp,
+               int32_t *__restrict__ wcnt, int32_t *__restrict__ Ccol, V *__restrict__ Cval)
 {
     extern __shared__ __align__(16) char spa_smem[];
     double *acc = reinterpret_cast<double *>(spa_smem);                       // [SPA_W] (numeric)
     uint32_t *mark = reinterpret_cast<uint32_t *>(spa_smem + (NUM ? SPA_W * 8 : 0));  // [SPA_W / 32]
     __shared__ int32_t wsum[SPA_NT / 32];
+    __shared__ int32_t s_r;
+    __shared__ int32_t s_qlo[SPA_NT], s_qhi[SPA_NT];  // each A nonzero's B entries inside the window
     const int tid = threadIdx.x;
-    const int32_t r = sparow[blockIdx.x];
-    const int32_t c0 = spanlo[r];
-    const int span = spanhi[r] - c0 + 1;
+    const int64_t item = blockIdx.x;
+    if (tid == 0) {  // the row owning this item: last r with spapos[r] <= item
+        int64_t lo = 0, hi = m;
+        while (hi - lo > 1) {
+            const int64_t mid = (lo + hi) >> 1;
+            if (spapos[mid] <= item) lo = mid;
+            else hi = mid;
+        }
+        while (lo + 1 < m && spapos[lo + 1] <= item) ++lo;  // rows without windows share the offset
+        s_r = int32_t(lo);
+    }
+    __syncthreads();
+    const int32_t r = s_r;
+    const int64_t win = item - spapos[r];
+    const int32_t c0 = int32_t(int64_t(spanlo[r]) + win * SPA_W);
+    const int span = int((int64_t(spanhi[r]) - c0 + 1 < SPA_W ? int64_t(spanhi[r]) - c0 + 1 : int64_t(SPA_W)));
+    const bool whole = (win == 0) && (int64_t(spanhi[r]) - spanlo[r] + 1 <= SPA_W);  // one window: no searches
     const int nw = (span + 31) >> 5;
     for (int i = tid; i < nw; i += SPA_NT) mark[i] = 0u;
     __syncthreads();
     const int32_t a0 = Arp[r], a1 = Arp[r + 1];
-    for (int32_t j = a0; j < a1; ++j) {
-        const int32_t k = Acol[j];
-        const int32_t b0 = Brp[k], b1 = Brp[k + 1];
+    for (int32_t jc = a0; jc < a1; jc += SPA_NT) {
+        // this chunk's A nonzeros: their B row ranges clipped to the window
+        if (jc + tid < a1) {
+            const int32_t k = Acol[jc + tid];
+            int32_t b0 = Brp[k], b1 = Brp[k + 1];
+            if (!whole) {
+                int32_t lo = b0, hi = b1;  // first entry >= c0
+                while (lo < hi) {
+                    const int32_t mid = (lo + hi) >> 1;
+                    if (Bcol[mid] < c0) lo = mid + 1;
+                    else hi = mid;
+                }
+                b0 = lo;
+                hi = b1;  // first entry >= c0 + span
+                while (lo < hi) {
+                    const int32_t mid = (lo + hi) >> 1;
+                    if (Bcol[mid] < c0 + span) lo = mid + 1;
+                    else hi = mid;
+                }
+                b1 = lo;
+            }
+            s_qlo[tid] = b0;
+            s_qhi[tid] = b1;
+        }
+        __syncthreads();
+        const int nj = min(SPA_NT, a1 - jc);
+    for (int32_t jj = 0; jj < nj; ++jj) {
+        const int32_t j = jc + jj;
+        const int32_t b0 = s_qlo[jj], b1 = s_qhi[jj];
         double a = 0.0;
         if constexpr (NUM) a = double(Aval[j]);
         for (int32_t q = b0 + tid; q < b1; q += SPA_NT) {
@@ -251,6 +301,8 @@ spa_row_kernel(const int32_t *__restrict__ sparow, const int32_t *__restrict__ A
         }
         if constexpr (NUM) __syncthreads();  // column sums advance in k order
     }
+        __syncthreads();  // the range buffers are refilled by the next chunk
+    }
     __syncthreads();
     // marked columns, ascending: thread t owns words [t*WPT, (t+1)*WPT)
     constexpr int WPT = (SPA_W / 32 + SPA_NT - 1) / SPA_NT;
@@ -263,9 +315,17 @@ spa_row_kernel(const int32_t *__restrict__ sparow, const int32_t *__restrict__ A
     int tot;
     int o = block_exclusive_sum<int, SPA_NT / 32>(cnt, wsum, 1, &tot);
     if constexpr (!NUM) {
-        if (tid == 0) Crp_counts[r] = tot;
+        if (tid == 0) {
+            wcnt[item] = tot;
+            atomicAdd(&Crp_counts[r], tot);
+        }
     } else {
-        const int64_t base = int64_t(Crp[r]) + o;
+        // output offset of this window: the row's earlier windows' counts
+        int pre = 0;
+        for (int64_t i = spapos[r] + tid; i < item; i += SPA_NT) pre += wcnt[i];
+        int pre_tot;
+        (void)block_exclusive_sum<int, SPA_NT / 32>(pre, wsum, 1, &pre_tot);
+        const int64_t base = int64_t(Crp[r]) + pre_tot + o;
         int64_t p = base;
 #pragma unroll
         for (int u = 0; u < WPT; ++u) {
@@ -1654,6 +1714,7 @@ struct MainWs {
     int32_t *ucol;   // row-accumulator path: each short row's output columns at its product offset
     int32_t *xcol;   // small-row path: B column of every product (symbolic expand; numeric reads it)
     double *xval;    // small-row path: every product a_ik * b_kj (numeric expand)
+    int32_t *spawcnt;  // segmented path: output count of every window (symbolic; numeric's offsets)
     int32_t *Xc[2];
     double *Xv[2];
     int32_t *heads;
@@ -1664,7 +1725,8 @@ struct MainWs {
     size_t bytes;
 };
 
-MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, int64_t nucol, int64_t nx, void *ws, size_t cap, bool *ok)
+MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, int64_t nucol, int64_t nx, int64_t nspa, void *ws,
+                  size_t cap, bool *ok)
 {
     MainWs w;
     Carve cv(ws, cap);
@@ -1673,6 +1735,7 @@ MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, int64_t nucol, int64_t 
     w.ucol = cv.take<int32_t>(size_t(nucol > 0 ? nucol : 1));
     w.xcol = cv.take<int32_t>(size_t(nx > 0 ? nx : 1));
     w.xval = cv.take<double>(size_t(nx > 0 ? nx : 1));
+    w.spawcnt = cv.take<int32_t>(size_t(nspa > 0 ? nspa : 1));
     for (int i = 0; i < 2; ++i) {
         w.Xc[i] = cv.take<int32_t>(size_t(LP > 0 ? LP : 1));
         w.Xv[i] = cv.take<double>(size_t(LP > 0 ? LP : 1));
@@ -1935,7 +1998,8 @@ bool spa_enabled()
 }
 
 template <typename V, bool NUM>
-msp_status run_spa(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const HostInfo &h, int32_t *Crp,
+msp_status run_spa(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, const HostInfo &h,
+                   int32_t *Crp,
                    int32_t *Ccol, void *Cval, cudaStream_t s)
 {
     if (h.nspa <= 0) return MSP_OK;
@@ -1943,10 +2007,11 @@ msp_status run_spa(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const 
     const int smem = (NUM ? SPA_W * 8 : 0) + SPA_W / 8 + 64;
     msp_status st = set_smem_attr(reinterpret_cast<const void *>(kern), smem, "spgemm: segmented smem");
     if (st != MSP_OK) return st;
-    kern<<<unsigned(h.nspa), SPA_NT, smem, s>>>(sw.sparow, A->row_offsets, A->col_idx,
+    kern<<<unsigned(h.nspa), SPA_NT, smem, s>>>(A->nrows, sw.spapos, A->row_offsets, A->col_idx,
                                                 static_cast<const V *>(A->vals), B->row_offsets, B->col_idx,
                                                 static_cast<const V *>(B->vals), sw.spanlo, sw.spanhi,
-                                                NUM ? nullptr : Crp + 1, Crp, Ccol, static_cast<V *>(Cval));
+                                                NUM ? nullptr : Crp + 1, Crp, mw.spawcnt, Ccol,
+                                                static_cast<V *>(Cval));
     return last_launch(NUM ? "spa_row_kernel<numeric>" : "spa_row_kernel<symbolic>");
 }
 
@@ -1964,7 +2029,7 @@ msp_status prepare_main(const msp_csr *A, const void *ws1, size_t b1, void *ws2,
     *sw = carve_setup(A, const_cast<void *>(ws1), b1, &ok1);
     if (!ok1) return MSP_ERR_WORKSPACE;
     *mw = carve_main(A->nrows, ntiles_of(A->nnz, h.nprods, h.rowacc), h.LP, h.nbitmap > 0 ? h.nprods : 0,
-                     h.nsmall > 0 ? h.nprods : 0, ws2, b2, &ok2);
+                     h.nsmall > 0 ? h.nprods : 0, h.nspa, ws2, b2, &ok2);
     if (!ok2) return MSP_ERR_WORKSPACE;
     return MSP_OK;
 }
@@ -2065,9 +2130,6 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
         if (st != MSP_OK) return st;
         st = scan_i32_to_i64(w.spaflag, w.spapos, m, w.scan, w.scan_bytes, s);
         if (st != MSP_OK) return st;
-        spa_scatter_kernel<<<blocks, 256, 0, s>>>(A->nrows, w.spaflag, w.spapos, w.sparow);
-        st = last_launch("spa_scatter_kernel");
-        if (st != MSP_OK) return st;
         st = scan_i32_to_i64(w.longflag, w.longpos, m, w.scan, w.scan_bytes, s);
         if (st != MSP_OK) return st;
         st = cuda_check(cudaMemsetAsync(w.longC, 0, size_t(m) * sizeof(int64_t), s), "spgemm: clear");
@@ -2091,8 +2153,8 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
     if (st != MSP_OK) return st;
     const int64_t ntiles = ntiles_of(nnz, h.nprods, h.rowacc);
     bool ok2;
-    MainWs mw = carve_main(m, ntiles, h.LP, h.nbitmap > 0 ? h.nprods : 0, h.nsmall > 0 ? h.nprods : 0, nullptr,
-                           SIZE_MAX, &ok2);
+    MainWs mw = carve_main(m, ntiles, h.LP, h.nbitmap > 0 ? h.nprods : 0, h.nsmall > 0 ? h.nprods : 0, h.nspa,
+                           nullptr, SIZE_MAX, &ok2);
     info->nprods = h.nprods;
     info->ntiles = ntiles;
     info->long_rows = h.nlong;
@@ -2166,8 +2228,8 @@ msp_status spgemm_pass(const msp_csr *A, const msp_csr *B, const void *ws1, size
         st = (A->dtype == MSP_F64) ? run_long<double, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s)
                                    : run_long<float, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s);
         if (st != MSP_OK) return st;
-        st = (A->dtype == MSP_F64) ? run_spa<double, NUM>(A, B, sw, h, Crp, Ccol, Cval, s)
-                                   : run_spa<float, NUM>(A, B, sw, h, Crp, Ccol, Cval, s);
+        st = (A->dtype == MSP_F64) ? run_spa<double, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s)
+                                   : run_spa<float, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s);
         if (st != MSP_OK) return st;
     }
     if (!NUM) {

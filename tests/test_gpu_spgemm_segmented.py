@@ -77,6 +77,40 @@ def test_mixed_rows():
     assert ok, msg
 
 
+def windowed(seed, mode="random"):
+    """long rows whose output span (60,000 columns) needs 5 windows of 12,288:
+    each A row references one long B row (30,000 entries over the span) and a
+    few short ones -- windows x nnz(row) = 5 x 5 <= ~30,000 products"""
+    g = np.random.default_rng(seed)
+    n, kb = 60_000, 400
+    brows = [np.sort(g.choice(n, 30_000, replace=False)) if k % 100 == 0 else np.unique(g.integers(0, n, 6))
+             for k in range(kb)]
+    brp = np.concatenate([[0], np.cumsum([x.size for x in brows])]).astype(np.int32)
+    bcol = np.concatenate(brows).astype(np.int32)
+    arows = [np.unique(np.concatenate([[100 * (r % 4)], g.integers(0, kb, 4)])) for r in range(120)]
+    arp = np.concatenate([[0], np.cumsum([x.size for x in arows])]).astype(np.int32)
+    acol = np.concatenate(arows).astype(np.int32)
+    if mode == "int":
+        return (gen.CSR(120, kb, arp, acol, gen.int_values(acol.size, seed)),
+                gen.CSR(kb, n, brp, bcol, gen.int_values(bcol.size, seed + 1)))
+    return (gen.CSR(120, kb, arp, acol, gen.matrices.random_values(acol.size, seed)),
+            gen.CSR(kb, n, brp, bcol, gen.matrices.random_values(bcol.size, seed + 1)))
+
+
+@pytest.mark.parametrize("mode", ["random", "int"])
+def test_windowed_wide_rows(mode):
+    """Spans wider than 12,288 columns cut into windows, one CTA each; a
+    window's output goes after the row's earlier windows' outputs."""
+    A, B = windowed(8, mode)
+    (rp, col, val), info = run(A, B)
+    W, sc, _ = oracle.spgemm(A, B)
+    spans = [(W.col[W.rp[r + 1] - 1] - W.col[W.rp[r]] + 1) for r in range(A.m)]
+    assert max(spans) > 4 * 12288
+    assert info.long_rows == 0 and info.segmented_rows > A.m  # several windows per row
+    assert np.array_equal(rp, W.rp) and np.array_equal(col, W.col)
+    assert np.array_equal(val, W.val), "k-ordered accumulation: bit-exact"
+
+
 _OFF = r"""
 import sys, numpy as np
 sys.path.insert(0, {root!r})
