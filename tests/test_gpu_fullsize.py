@@ -5,7 +5,8 @@ configuration bench.py times) and the boundary's error paths on the GPU.
   value within tau * sum_k |a_ik||b_kj| (BJ:5, Z18) against Gustavson's
   oracle on the whole matrix (not sampled rows).
 * SpMV / SpAdd C3 (R-MAT scale 22, fp32) at full size; SpMV C5 (10^8 rows)
-  at full size.
+  at full size; SpGEMM C5 A*A at full size (invariants on every row, 3,000
+  sampled rows exact against the oracle).
 * The 64-bit-key SpGEMM tile path (tiles whose row span does not fit the
   32-bit packed key next to the column bits), forced by construction.
 * msp_csr_check, MSP_ERR_INPUT (unsorted set-operation keys, malformed CSR
@@ -139,6 +140,46 @@ def test_c5_spmv_full():
     x = gen.x_vector(A.n, "int")
     y = spmv(dev(A), torch.as_tensor(x, device="cuda")).cpu().numpy()
     assert np.array_equal(y, oracle.spmv(A, x)[0])
+
+
+def test_c5_spgemm_full_sampled():
+    """C5 A*A (BJ:11) at full size: 1.6e9 products through the small-row
+    path.  On the GPU: Nprods, every row's length <= its product count and
+    its columns strictly increasing, C.row_offsets consistent; 3,000 rows
+    spread over the matrix (plus the first and last) against Gustavson's
+    oracle, exact (integer mode)."""
+    import torch
+    from paper_conf_ipps_daltonbmog15_b200 import SpGemmPlan
+    A = gen.config("C5", "int")
+    blen = np.diff(A.rp.astype(np.int64))
+    pa = blen[A.col]
+    cs = np.zeros(A.nnz + 1, np.int64)
+    np.cumsum(pa, out=cs[1:])
+    P = cs[A.rp[1:]] - cs[A.rp[:-1]]
+    del pa, cs
+    dA = dev(A)
+    p = SpGemmPlan(dA, dA)
+    info = p.setup()
+    assert info.nprods == int(P.sum())
+    C = p.numeric()
+    assert info.small_rows == int(np.count_nonzero((P > 0) & (P <= 64))) and info.ntiles == 0
+    rp = C.rp.to(torch.int64)
+    lens = rp[1:] - rp[:-1]
+    assert int(rp[0]) == 0 and bool((lens >= 0).all()) and int(rp[-1]) == C.nnz
+    assert bool((lens <= torch.as_tensor(P, device="cuda")).all())
+    col = C.col.to(torch.int64)
+    inc = col[1:] > col[:-1]
+    starts = rp[1:-1][lens[1:] > 0]  # first entry of every nonempty row after the first
+    inc[starts - 1] = True
+    assert bool(inc.all()), "columns not strictly increasing inside a row"
+    rows = np.unique(np.concatenate([[0, A.m - 1], np.random.default_rng(7).integers(0, A.m, 3000)]))
+    off, wcol, wval, _ = oracle.spgemm_rows(A, A, rows)
+    rph = C.rp.cpu().numpy()
+    for k, r in enumerate(rows):
+        a, b = int(rph[r]), int(rph[r + 1])
+        assert b - a == off[k + 1] - off[k], f"row {r}: length"
+        assert np.array_equal(C.col[a:b].cpu().numpy(), wcol[off[k]:off[k + 1]]), f"row {r}: columns"
+        assert np.array_equal(C.val[a:b].cpu().numpy(), wval[off[k]:off[k + 1]]), f"row {r}: values"
 
 
 # ------------------------------------------------------------- error paths
