@@ -78,9 +78,12 @@ struct CtaRecord {  // one per CTA in the workspace
 
 // NW worker warps of 32 lanes x K = 8 products each (one tile = NW * 256
 // merge items), plus one producer warp and one row warp.
-template <typename V, int NW_, int STAGES_, int RSLOTS_, int MINB_, bool EARLY_ = false>
+template <typename V, int NW_, int STAGES_, int RSLOTS_, int MINB_, bool EARLY_ = false, bool L1G_ = false>
 struct Cfg {
     static constexpr bool ROWK = false;
+    // L1G: x gathers allocate in L1 (ld.global.nc.L2::64B): R-MAT hub columns
+    // are reused (C3 419 -> 407 us); else L2 only (ld.global.cg.L2::64B)
+    static constexpr bool L1G = L1G_;
     // EARLY: a worker issues tile t+1's x gathers right after forming tile
     // t's products (they fly during t's walk, scan and look-back) instead of
     // after the walk
@@ -195,9 +198,22 @@ __device__ __forceinline__ double ldg_x(const float *p)
 #ifndef MSP_SPMV_GATHER
 #define MSP_SPMV_GATHER 3
 #endif
-template <typename T>
+template <typename T, bool L1G = false>
 __device__ __forceinline__ T gather_x(const T *p)
 {
+    if constexpr (L1G) {
+        T v;
+        if constexpr (sizeof(T) == 8) {
+            double d;
+            asm volatile("ld.global.nc.L2::64B.f64 %0, [%1];" : "=d"(d) : "l"(p));
+            v = T(d);
+        } else {
+            float f;
+            asm volatile("ld.global.nc.L2::64B.f32 %0, [%1];" : "=f"(f) : "l"(p));
+            v = T(f);
+        }
+        return v;
+    }
 #if MSP_SPMV_GATHER == 1
     return __ldcg(p);
 #elif MSP_SPMV_GATHER == 2
@@ -723,7 +739,7 @@ spmv_merge_kernel(int32_t m, int64_t nnz, const int32_t *__restrict__ rp, const 
                 cidx[u] = int(c < col_lim ? c : 0u);
             }
 #pragma unroll
-            for (int u = 0; u < K; ++u) xv[u] = gather_x(x + cidx[u]);
+            for (int u = 0; u < K; ++u) xv[u] = gather_x<V, C::L1G>(x + cidx[u]);
 #pragma unroll
             for (int u = 0; u < K; ++u) vv[u] = vs[lane + 32 * u];
         };
@@ -947,7 +963,7 @@ template <typename V> struct Shape<V, 5> { using C = Cfg<V, 4, 2, 4, 5>; };
 template <typename V> struct Shape<V, 6> { using C = Cfg<V, 2, 2, 4, 8>; };
 template <typename V> struct Shape<V, 7> { using C = Cfg<V, 2, 2, 4, 6>; };
 template <typename V> struct Shape<V, 8> { using C = Cfg<V, 4, 2, 4, 4, true>; };
-template <typename V> struct Shape<V, 9> { using C = Cfg<V, 2, 2, 4, 8, true>; };
+template <typename V> struct Shape<V, 9> { using C = Cfg<V, 2, 2, 4, 8, true, true>; };
 template <typename V> struct Shape<V, 10> { using C = Cfg<V, 2, 3, 4, 8, true>; };
 template <typename V> struct Shape<V, 11> { using C = Cfg<V, 2, 4, 4, 8, true>; };
 constexpr int kNumShapes = 12;
