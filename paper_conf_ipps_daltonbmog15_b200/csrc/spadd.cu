@@ -204,33 +204,57 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
     const int ga0 = s0.a, gb0 = s0.b;
     const int nA = s1.a - ga0, nB = s1.b - gb0;
     const int nrw = min(r1, m - 1) - r0 + 2;  // row offsets r0 .. min(r1, m-1)+1
-    if (tid == 0) {
-        mbar_init(bar, 1);
-        fence_mbar_init();
-    }
-    __syncthreads();
     // ---- stage the tile: one TMA bulk copy per window ----
-    const uint64_t pol = policy_evict_first();
-    int ioff = 0, voff = L::V_OFF;
-    uint32_t tx = 0;
-    const Staged p_arp = plan_stage<int32_t>(Arp, r0, r0 + nrw, int64_t(m) + 1, &ioff, &tx);
-    const Staged p_brp = plan_stage<int32_t>(Brp, r0, r0 + nrw, int64_t(m) + 1, &ioff, &tx);
-    const Staged p_ac = plan_stage<int32_t>(Acol, ga0, ga0 + nA, nnzA, &ioff, &tx);
-    const Staged p_bc = plan_stage<int32_t>(Bcol, gb0, gb0 + nB, nnzB, &ioff, &tx);
-    Staged p_av{}, p_bv{};
-    if constexpr (FILL) {
-        p_av = plan_stage<V>(Aval, ga0, ga0 + nA, nnzA, &voff, &tx);
-        p_bv = plan_stage<V>(Bval, gb0, gb0 + nB, nnzB, &voff, &tx);
+    // Warp 0 plans the windows (the other warps only need their shared-memory
+    // offsets, published with the barrier below) and copies their ragged ends.
+    __shared__ int s_first[6];
+    if (tid < 32) {
+        if (tid == 0) {
+            mbar_init(bar, 1);
+            fence_mbar_init();
+        }
+        __syncwarp();
+        const uint64_t pol = policy_evict_first();
+        int ioff = 0, voff = L::V_OFF;
+        uint32_t tx = 0;
+        const Staged p_arp = plan_stage<int32_t>(Arp, r0, r0 + nrw, int64_t(m) + 1, &ioff, &tx);
+        const Staged p_brp = plan_stage<int32_t>(Brp, r0, r0 + nrw, int64_t(m) + 1, &ioff, &tx);
+        const Staged p_ac = plan_stage<int32_t>(Acol, ga0, ga0 + nA, nnzA, &ioff, &tx);
+        const Staged p_bc = plan_stage<int32_t>(Bcol, gb0, gb0 + nB, nnzB, &ioff, &tx);
+        Staged p_av{}, p_bv{};
+        if constexpr (FILL) {
+            p_av = plan_stage<V>(Aval, ga0, ga0 + nA, nnzA, &voff, &tx);
+            p_bv = plan_stage<V>(Bval, gb0, gb0 + nB, nnzB, &voff, &tx);
+        }
+        if (tid == 0) mbar_arrive_expect_tx(bar, tx);
+        int32_t *w_arp = issue_stage<int32_t>(p_arp, Arp, r0, r0 + nrw, smem_raw, bar, 0);
+        int32_t *w_brp = issue_stage<int32_t>(p_brp, Brp, r0, r0 + nrw, smem_raw, bar, 0);
+        const int32_t *w_ac = issue_stage<int32_t>(p_ac, Acol, ga0, ga0 + nA, smem_raw, bar, pol);
+        const int32_t *w_bc = issue_stage<int32_t>(p_bc, Bcol, gb0, gb0 + nB, smem_raw, bar, pol);
+        if (tid == 0) {
+            s_first[0] = int(reinterpret_cast<char *>(w_arp) - smem_raw);
+            s_first[1] = int(reinterpret_cast<char *>(w_brp) - smem_raw);
+            s_first[2] = int(reinterpret_cast<const char *>(w_ac) - smem_raw);
+            s_first[3] = int(reinterpret_cast<const char *>(w_bc) - smem_raw);
+        }
+        if constexpr (FILL) {
+            const V *w_av = issue_stage<V>(p_av, Aval, ga0, ga0 + nA, smem_raw, bar, pol);
+            const V *w_bv = issue_stage<V>(p_bv, Bval, gb0, gb0 + nB, smem_raw, bar, pol);
+            if (tid == 0) {
+                s_first[4] = int(reinterpret_cast<const char *>(w_av) - smem_raw);
+                s_first[5] = int(reinterpret_cast<const char *>(w_bv) - smem_raw);
+            }
+        }
     }
-    if (tid == 0) mbar_arrive_expect_tx(bar, tx);
-    int32_t *arp = issue_stage<int32_t>(p_arp, Arp, r0, r0 + nrw, smem_raw, bar, 0);
-    int32_t *brp = issue_stage<int32_t>(p_brp, Brp, r0, r0 + nrw, smem_raw, bar, 0);
-    const int32_t *acs = issue_stage<int32_t>(p_ac, Acol, ga0, ga0 + nA, smem_raw, bar, pol);
-    const int32_t *bcs = issue_stage<int32_t>(p_bc, Bcol, gb0, gb0 + nB, smem_raw, bar, pol);
+    __syncthreads();  // mbarrier initialised, window offsets published
+    int32_t *arp = reinterpret_cast<int32_t *>(smem_raw + s_first[0]);
+    int32_t *brp = reinterpret_cast<int32_t *>(smem_raw + s_first[1]);
+    const int32_t *acs = reinterpret_cast<const int32_t *>(smem_raw + s_first[2]);
+    const int32_t *bcs = reinterpret_cast<const int32_t *>(smem_raw + s_first[3]);
     const V *avs = nullptr, *bvs = nullptr;
     if constexpr (FILL) {
-        avs = issue_stage<V>(p_av, Aval, ga0, ga0 + nA, smem_raw, bar, pol);
-        bvs = issue_stage<V>(p_bv, Bval, gb0, gb0 + nB, smem_raw, bar, pol);
+        avs = reinterpret_cast<const V *>(smem_raw + s_first[4]);
+        bvs = reinterpret_cast<const V *>(smem_raw + s_first[5]);
     }
     mbar_wait(bar, 0);
     __syncthreads();  // ragged ends written by warp 0
@@ -471,8 +495,10 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
             __syncthreads();
             // the tile's run of C is contiguous: coalesced stores
             const int64_t base = tbase;
-            const int nst = min(tot, ADD_T);  // binds only on malformed input
-            for (int i = tid; i < nst && base + i < cap; i += ADD_NT) {
+            // min(tot, ADD_T) and the capacity bind only on malformed input
+            const int64_t room = cap - base > 0 ? cap - base : 0;
+            const int nst = int(room < int64_t(min(tot, ADD_T)) ? room : int64_t(min(tot, ADD_T)));
+            for (int i = tid; i < nst; i += ADD_NT) {
                 Ccol[base + i] = ocol[i];
                 Cval[base + i] = oval[i];
             }
