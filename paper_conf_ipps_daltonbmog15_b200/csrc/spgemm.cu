@@ -501,6 +501,14 @@ __global__ void wr_class_kernel(int32_t m, const int32_t *__restrict__ Arp, cons
 //     roundings -- and (c, sum) goes to C.rp[r] + rank.
 // O(P_r) work per product, cheap for small rows; no sort.
 constexpr int WS_WARPS = 4;
+// WS_RANKS=1 (experiment): symbolic computes every product's rank in its row
+// (smaller columns, one loop) and stores it as a byte next to the staged
+// products, so numeric writes duplicate-free rows without a loop.  Measured on
+// C5: symbolic compress 12.7 -> 24.2 ms, numeric 17.9 -> 12.1 ms (net slower);
+// default 0: the symbolic hash count and the numeric rank loop.
+#ifndef WS_RANKS
+#define WS_RANKS 0
+#endif
 #ifndef WS_PAD
 #define WS_PAD 0
 #endif
@@ -549,7 +557,8 @@ template <typename V, bool NUM>
 __global__ void __launch_bounds__(WS_WARPS * 32, (NUM && WS_PAD) ? 6 : 8)
 ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__restrict__ wmode,
                 const int64_t *__restrict__ S, const int32_t *__restrict__ X, const double *__restrict__ XV,
-                int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol, V *__restrict__ Cval)
+                uint8_t *__restrict__ XR, int32_t *__restrict__ Crp, int32_t *__restrict__ Ccol,
+                V *__restrict__ Cval)
 {
     constexpr unsigned FULL = 0xffffffffu;
     // WS_PAD (experiment): numeric stores each row at a 4-aligned start padded
@@ -562,20 +571,22 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__res
     __shared__ int16_t s_slot_all[NUM ? 1 : WS_WARPS][NUM ? 1 : WS_BATCH];  // symbolic: hash slot of each product
     __shared__ unsigned s_first_all[NUM ? WS_WARPS : 1][KCAP / 32];         // numeric: first-occurrence bits
     __shared__ int s_cnt_all[WS_WARPS][32];                                   // symbolic: duplicates per row
-    __shared__ unsigned long long s_hash_all[NUM ? 1 : WS_WARPS][NUM ? 1 : WS_HASH];  // symbolic: (row, col) set
+    __shared__ unsigned long long s_hash_all[(NUM || WS_RANKS) ? 1 : WS_WARPS][(NUM || WS_RANKS) ? 1 : WS_HASH];
     __shared__ double s_val_all[NUM ? WS_WARPS : 1][NUM ? KCAP : 1];
+    __shared__ uint8_t s_rank_all[(NUM && WS_RANKS) ? WS_WARPS : 1][(NUM && WS_RANKS) ? WS_BATCH : 1];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     int32_t *s_key = s_key_all[warp];
     uint8_t *s_row = s_row_all[warp];
     int16_t *s_slot = s_slot_all[NUM ? 0 : warp];
-    unsigned long long *s_hash = s_hash_all[NUM ? 0 : warp];
+    unsigned long long *s_hash = s_hash_all[(NUM || WS_RANKS) ? 0 : warp];
     unsigned *s_first = s_first_all[NUM ? warp : 0];
     int *s_cnt = s_cnt_all[warp];
     double *s_val = s_val_all[NUM ? warp : 0];
+    uint8_t *s_rank = s_rank_all[(NUM && WS_RANKS) ? warp : 0];
     const int64_t nwarps = int64_t(gridDim.x) * WS_WARPS;
     s_cnt[lane] = 0;
     reinterpret_cast<uint2 *>(s_row)[lane] = make_uint2(0u, 0u);
-    if constexpr (!NUM)
+    if constexpr (!NUM && !WS_RANKS)
         for (int i = lane; i < WS_HASH; i += 32) s_hash[i] = WS_EMPTY;
     for (int64_t r0 = (int64_t(blockIdx.x) * WS_WARPS + warp) * 32; r0 < m; r0 += nwarps * 32) {
         const int64_t r = r0 + lane;
@@ -608,11 +619,13 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__res
             // ---- the batch's staged products: coalesced, all loads in flight ----
             int32_t ck[WS_PPL];
             double cv[WS_PPL];
+            uint32_t crk[WS_PPL];
 #pragma unroll
             for (int u = 0; u < WS_PPL; ++u) {
                 const int p = u * 32 + lane;
                 ck[u] = p < np ? X[base + p] : 0;
                 if constexpr (NUM) cv[u] = p < np ? XV[base + p] : 0.0;
+                if constexpr (NUM && WS_RANKS) crk[u] = p < np ? XR[base + p] : 0u;
             }
             // ---- row lane of every position: start marks, blocked max-scan ----
             if (inb) s_row[prel] = uint8_t(lane + 1);
@@ -659,6 +672,7 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__res
                 if (p < np) {
                     s_key[pp] = ck[u];
                     if constexpr (NUM) s_val[pp] = cv[u];
+                    if constexpr (NUM && WS_RANKS) s_rank[p] = uint8_t(crk[u]);
                 }
             }
             __syncwarp();
@@ -668,7 +682,25 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__res
                 const int p = pr + lane;
                 const bool act = p < np;
                 const int t = act ? int(s_row[p]) : s;  // the product's row lane
-                if constexpr (!NUM) {
+                if constexpr (!NUM && WS_RANKS) {
+                    // one loop over the row: the product's rank (smaller
+                    // columns) for numeric, and whether an earlier product of
+                    // the row has the same column (a duplicate, not counted)
+                    const int seg = __shfl_sync(FULL, prel, t);
+                    const int len = __shfl_sync(FULL, P, t);
+                    if (act) {
+                        const int32_t c = s_key[p];
+                        int less = 0;
+                        bool dup = false;
+                        for (int q = seg; q < seg + len; ++q) {
+                            const int32_t kq = s_key[q];
+                            less += kq < c ? 1 : 0;
+                            dup = dup || (kq == c && q < p);
+                        }
+                        XR[base + p] = uint8_t(less);
+                        if (dup) atomicAdd(&s_cnt[t], 1);
+                    }
+                } else if constexpr (!NUM) {
                     // distinct (row, column) pairs: insert into the warp's hash
                     // set; an insert that finds its own key is a duplicate
                     if (act) {
@@ -697,7 +729,9 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__res
                         // rank = smaller columns in the row (4 per shared load; pads never count)
                         const int32_t c = s_key[pp];
                         int rk = 0;
-                        if constexpr (PADDED) {
+                        if constexpr (WS_RANKS) {
+                            rk = s_rank[p];  // from symbolic
+                        } else if constexpr (PADDED) {
                             for (int q = seg; q < seg + len; q += 4) {
                                 const int4 w = *reinterpret_cast<const int4 *>(s_key + q);
                                 rk += int(w.x < c) + int(w.y < c) + int(w.z < c) + int(w.w < c);
@@ -710,7 +744,7 @@ ws_small_kernel(int32_t m, const int32_t *__restrict__ Arp, const uint8_t *__res
                     }
                 }
             }
-            if constexpr (!NUM) {
+            if constexpr (!NUM && !WS_RANKS) {
                 // clear the slots this batch used (a duplicate's probe ends on
                 // its first occurrence's slot: cleared twice, harmlessly)
                 __syncwarp();
@@ -1714,6 +1748,7 @@ struct MainWs {
     int32_t *ucol;   // row-accumulator path: each short row's output columns at its product offset
     int32_t *xcol;   // small-row path: B column of every product (symbolic expand; numeric reads it)
     double *xval;    // small-row path: every product a_ik * b_kj (numeric expand)
+    uint8_t *xrank;  // small-row path: every product's rank in its row (symbolic compress)
     int32_t *spawcnt;  // segmented path: output count of every window (symbolic; numeric's offsets)
     int32_t *Xc[2];
     double *Xv[2];
@@ -1735,6 +1770,7 @@ MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, int64_t nucol, int64_t 
     w.ucol = cv.take<int32_t>(size_t(nucol > 0 ? nucol : 1));
     w.xcol = cv.take<int32_t>(size_t(nx > 0 ? nx : 1));
     w.xval = cv.take<double>(size_t(nx > 0 ? nx : 1));
+    w.xrank = cv.take<uint8_t>(size_t(nx > 0 ? nx : 1));
     w.spawcnt = cv.take<int32_t>(size_t(nspa > 0 ? nspa : 1));
     for (int i = 0; i < 2; ++i) {
         w.Xc[i] = cv.take<int32_t>(size_t(LP > 0 ? LP : 1));
@@ -1924,8 +1960,8 @@ msp_status run_small(const msp_csr *A, const msp_csr *B, const SetupWs &sw, cons
     if (st != MSP_OK) return st;
     const int32_t m = A->nrows;
     const int64_t g = std::min<int64_t>(int64_t(occ) * sm_count(), ceil_div(m, WS_WARPS * 32));
-    kern<<<unsigned(g > 0 ? g : 1), WS_WARPS * 32, 0, s>>>(m, A->row_offsets, sw.wmode, sw.S, mw.xcol, mw.xval, Crp,
-                                                          Ccol, static_cast<V *>(Cval));
+    kern<<<unsigned(g > 0 ? g : 1), WS_WARPS * 32, 0, s>>>(m, A->row_offsets, sw.wmode, sw.S, mw.xcol, mw.xval,
+                                                          mw.xrank, Crp, Ccol, static_cast<V *>(Cval));
     return last_launch(NUM ? "ws_small_kernel<numeric>" : "ws_small_kernel<symbolic>");
 }
 
