@@ -1770,7 +1770,7 @@ MainWs carve_main(int64_t m, int64_t ntiles, int64_t LP, int64_t nucol, int64_t 
     w.ucol = cv.take<int32_t>(size_t(nucol > 0 ? nucol : 1));
     w.xcol = cv.take<int32_t>(size_t(nx > 0 ? nx : 1));
     w.xval = cv.take<double>(size_t(nx > 0 ? nx : 1));
-    w.xrank = cv.take<uint8_t>(size_t(nx > 0 ? nx : 1));
+    w.xrank = cv.take<uint8_t>(size_t((WS_RANKS && nx > 0) ? nx : 1));
     w.spawcnt = cv.take<int32_t>(size_t(nspa > 0 ? nspa : 1));
     for (int i = 0; i < 2; ++i) {
         w.Xc[i] = cv.take<int32_t>(size_t(LP > 0 ? LP : 1));
