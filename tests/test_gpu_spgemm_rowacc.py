@@ -113,7 +113,7 @@ def test_not_taken_on_wide_rows():
     assert info.row_accumulator == 0 and info.ntiles > 0
 
 
-_ESC_SUITE = ["tests/test_gpu_spgemm.py", "tests/test_gpu_spgemm_segmented.py"]
+_ESC_SUITE = ["tests/test_gpu_spgemm.py", "tests/test_gpu_spgemm_segmented.py", "tests/test_gpu_spgemm_fuzz.py"]
 
 
 @pytest.mark.skipif(os.environ.get("MSP_SPGEMM_ROWACC") == "0", reason="already the ESC-only run")
