@@ -2134,12 +2134,12 @@ msp_status spgemm_setup_run(const msp_csr *A, const msp_csr *B, void *ws1, size_
             st = last_launch("wr_class_kernel");
             if (st != MSP_OK) return st;
         }
-        // Large matrices: one extra synchronisation reads the long-row count
+        // Matrices with >= 1024 rows: one extra synchronisation reads the long-row count
         // (from the classification and the promotions); without long rows the
         // global-phase bookkeeping (spans, segmented classification, four
         // row scans, scatters) is skipped -- C5: ~4.7 ms of setup.
         bool any_long = true;
-        if (m >= (1 << 20)) {
+        if (m >= 1024) {
             int64_t v[13];
             st = read_back(reinterpret_cast<const int64_t *>(w.stats), 13, v, s, "spgemm: long rows");
             if (st != MSP_OK) return st;
