@@ -363,7 +363,10 @@ spa_row_kernel(int32_t m, const int64_t *__restrict__ spapos, const int32_t *__r
 // and add roundings, as the oracle does.  The choice is global (all short
 // rows or none) so that the tile pass is either skipped or untouched.
 constexpr int WR_SPAN = 65536;            // widest short-row span the bitmaps cover (8 KB per warp)
-constexpr int WR_SYM_WARPS = 8;           // 64 KB of bitmaps per CTA
+constexpr int WR_SYM_WARPS = 8;
+#ifndef WR_EMIT_SERIAL
+#define WR_EMIT_SERIAL 0  // experiment: per-lane serial emission of the column list
+#endif           // 64 KB of bitmaps per CTA
 constexpr int WR_UMAX = 512;              // accumulator entries per warp per pass (6 KB with the column list)
 constexpr int WR_NUM_WARPS = 8;
 
@@ -911,6 +914,24 @@ wr_symbolic_kernel(int32_t m, int nw_max, const int32_t *__restrict__ Arp, const
             const int p0 = __popc(w4.x), p1 = __popc(w4.y), p2 = __popc(w4.z), p3 = __popc(w4.w);
             int tot;
             const int ex = warp_excl_sum(p0 + p1 + p2 + p3, lane, &tot);
+#if WR_EMIT_SERIAL
+            // each lane emits its own words' set bits in order at ex + i
+            // (lanes' runs are adjacent: the stores stay within a few lines)
+            {
+                int pos = run + ex;
+                const uint32_t wv[4] = {w4.x, w4.y, w4.z, w4.w};
+#pragma unroll
+                for (int e = 0; e < 4; ++e) {
+                    uint32_t bits = wv[e];
+                    const int cbase = lo + (q * 128 + lane * 4 + e) * 32;
+                    while (bits) {
+                        const int bt = __ffs(bits) - 1;
+                        bits &= bits - 1;
+                        dst[pos++] = cbase + bt;
+                    }
+                }
+            }
+#else
             // the round's tot columns go out converged and coalesced: output o
             // (o = lane, lane + 32, ...) finds the lane owning it (last lane
             // with ex <= o), the word within that lane's four, and the bit
@@ -935,6 +956,7 @@ wr_symbolic_kernel(int32_t m, int nw_max, const int32_t *__restrict__ Arp, const
                 const int b = nth_set_bit(word, nth);
                 if (o < tot) dst[run + o] = lo + (q * 128 + src_l * 4 + e) * 32 + b;
             }
+#endif
             run += tot;
         }
         if (lane == 0) Crp_counts[r] = run;
