@@ -516,9 +516,16 @@ msp_status launch_wt(const msp_csr *A, const void *x, void *y, void *ws, size_t 
 {
     // 11 workers + the producer: 12 warps = 3 per SM sub-partition, so up to
     // 168 registers per thread (each sub-partition holds 16K registers);
-    // 3 stages of up to 8 warp tiles (about 62 KB each)
-    constexpr int NSUB0 = (188 * 1024 / 3) / int((4 + sizeof(V)) * 32 * K);
-    using C = WtCfg<V, K, 11, (NSUB0 < 24 ? NSUB0 : 24), 3>;
+    // 4 stages of warp tiles (about 47 KB each; 4 x 4 tiles for K = 27 fp64)
+#ifndef MSP_WT_STAGES  // tuning builds: ring depth and tiles per stage
+#define MSP_WT_STAGES 4  // C2: 4 x 4 warp tiles 68.4 us vs 3 x 6 70.7 us (profiles/r2/spmv_wt_ring_sweep.txt)
+#endif
+#ifndef MSP_WT_NSUB
+#define MSP_WT_NSUB 0  // 0: as many warp tiles as fit ~188 KB over the stages
+#endif
+    constexpr int NSUB0 = MSP_WT_NSUB > 0 ? MSP_WT_NSUB
+                                          : (188 * 1024 / MSP_WT_STAGES) / int((4 + sizeof(V)) * 32 * K);
+    using C = WtCfg<V, K, 11, (NSUB0 < 24 ? NSUB0 : 24), MSP_WT_STAGES>;
     auto kern = spmv_wt_kernel<V, C>;
     int occ = 1;
     static const bool fit = getenv("MSP_SPMV_WT_L1") != nullptr;  // experiment: carveout fitted to the CTA
