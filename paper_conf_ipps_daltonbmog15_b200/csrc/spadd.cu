@@ -39,7 +39,10 @@
 namespace msp {
 namespace {
 
-constexpr int ADD_NT = 256;
+#ifndef MSP_ADD_NT
+#define MSP_ADD_NT 128  // threads per tile: C3 one pass 0.880 -> 0.865 ms, C2 0.410 -> 0.389 ms vs 256 (64-512 swept)
+#endif
+constexpr int ADD_NT = MSP_ADD_NT;
 #ifndef MSP_ADD_IPT
 #define MSP_ADD_IPT 14  // measured on B200 (one-walk fill, 53-66 KB smem): C3 A+A^T 1.85 ms at 8, 1.42 at 12,
                         // 1.30 at 14, 1.31 at 16, 1.23 at 20; C2 0.47-0.49 ms at 12-20
