@@ -363,12 +363,21 @@ spa_row_kernel(int32_t m, const int64_t *__restrict__ spapos, const int32_t *__r
 // and add roundings, as the oracle does.  The choice is global (all short
 // rows or none) so that the tile pass is either skipped or untouched.
 constexpr int WR_SPAN = 65536;            // widest short-row span the bitmaps cover (8 KB per warp)
-constexpr int WR_SYM_WARPS = 8;
+#ifndef MSP_WR_SYM_WARPS  // tuning builds
+#define MSP_WR_SYM_WARPS 8
+#endif
+#ifndef MSP_WR_NUM_WARPS
+#define MSP_WR_NUM_WARPS 8
+#endif
+#ifndef MSP_WR_NUM_MINB
+#define MSP_WR_NUM_MINB 3
+#endif
+constexpr int WR_SYM_WARPS = MSP_WR_SYM_WARPS;
 #ifndef WR_EMIT_SERIAL
 #define WR_EMIT_SERIAL 0  // experiment: per-lane serial emission of the column list (C2 symbolic 2.25 -> 3.12 ms: slower)
 #endif           // 64 KB of bitmaps per CTA
 constexpr int WR_UMAX = 512;              // accumulator entries per warp per pass (6 KB with the column list)
-constexpr int WR_NUM_WARPS = 8;
+constexpr int WR_NUM_WARPS = MSP_WR_NUM_WARPS;
 
 __device__ __forceinline__ int warp_excl_sum(int v, int lane, int *total)
 {
@@ -503,7 +512,10 @@ __global__ void wr_class_kernel(int32_t m, const int32_t *__restrict__ Arp, cons
 //     products in position (= k) order -- the oracle's order, separate
 //     roundings -- and (c, sum) goes to C.rp[r] + rank.
 // O(P_r) work per product, cheap for small rows; no sort.
-constexpr int WS_WARPS = 4;
+#ifndef MSP_WS_WARPS
+#define MSP_WS_WARPS 4
+#endif
+constexpr int WS_WARPS = MSP_WS_WARPS;
 // WS_RANKS=1 (experiment): symbolic computes every product's rank in its row
 // (smaller columns, one loop) and stores it as a byte next to the staged
 // products, so numeric writes duplicate-free rows without a loop.  Measured on
@@ -976,7 +988,7 @@ __device__ __forceinline__ uint32_t wr_hash(uint32_t x) { return (x * 0x9E3779B1
 static_assert(WR_HSLOTS == 1024, "wr_hash yields 10 bits");
 
 template <typename V>
-__global__ void __launch_bounds__(WR_NUM_WARPS * 32, 3)
+__global__ void __launch_bounds__(WR_NUM_WARPS * 32, MSP_WR_NUM_MINB)
 wr_numeric_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__restrict__ Acol,
                   const V *__restrict__ Aval, const int32_t *__restrict__ Brp, const int32_t *__restrict__ Bcol,
                   const V *__restrict__ Bval, const uint8_t *__restrict__ wmode, const int64_t *__restrict__ S,
