@@ -5,7 +5,7 @@
 // P:820-822), and the SpGEMM product prefix S over the B row lengths
 // referenced by A's columns (reading Z8: a flat int64 exclusive
 // scan so that it can be binary-searched).  One pass: each CTA scans a
-// 4096-item tile warp-striped (coalesced loads/stores), publishes its
+// 2048-item tile warp-striped (coalesced loads/stores), publishes its
 // aggregate, and warp 0 looks back over its predecessors' published
 // (flag, value) words to obtain the tile prefix.  Accumulation is int64.
 #include "common.cuh"
@@ -15,7 +15,10 @@ namespace msp {
 namespace {
 
 constexpr int SCAN_NT = 256;
-constexpr int SCAN_ITEMS = 16;
+#ifndef MSP_SCAN_ITEMS
+#define MSP_SCAN_ITEMS 8  // 2,048-item tiles: C5 SpGEMM setup 14.9 -> 13.6 ms vs 16 (4-32 swept, profiles/r2/scan_items_sweep.txt)
+#endif
+constexpr int SCAN_ITEMS = MSP_SCAN_ITEMS;
 constexpr int SCAN_TILE = SCAN_NT * SCAN_ITEMS;
 constexpr unsigned long long FLAG_AGG = 1ull << 62;
 constexpr unsigned long long FLAG_INC = 2ull << 62;
