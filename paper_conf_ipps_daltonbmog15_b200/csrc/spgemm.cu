@@ -537,11 +537,13 @@ __global__ void __launch_bounds__(256)
 ws_expand_kernel(int64_t nnzA, const int32_t *__restrict__ arow, const uint8_t *__restrict__ wmode,
                  const int64_t *__restrict__ S, const int32_t *__restrict__ bstart, const V *__restrict__ Aval,
                  const int32_t *__restrict__ Bcol, const V *__restrict__ Bval, int32_t *__restrict__ X,
-                 double *__restrict__ XV)
+                 double *__restrict__ XV, int all_small)
 {
     const int64_t stride = int64_t(gridDim.x) * blockDim.x;
     for (int64_t j = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; j < nnzA; j += stride) {
-        if (wmode[arow[j]] != WM_SMALL) continue;
+        // (every row with products small -- C5 -- needs no row lookup: the
+        // nonzeros of other rows expand to nothing)
+        if (!all_small && wmode[arow[j]] != WM_SMALL) continue;
         const int64_t s0 = S[j];
         const int len = int(S[j + 1] - s0);
         const int32_t b0 = bstart[j];
@@ -1979,13 +1981,14 @@ bool small_enabled()
 }
 
 template <typename V, bool NUM>
-msp_status run_small(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, int32_t *Crp,
-                     int32_t *Ccol, void *Cval, cudaStream_t s)
+msp_status run_small(const msp_csr *A, const msp_csr *B, const SetupWs &sw, const MainWs &mw, const HostInfo &h,
+                     int32_t *Crp, int32_t *Ccol, void *Cval, cudaStream_t s)
 {
     const int64_t nnz = A->nnz;
+    const int all_small = (h.nbitmap == 0 && h.nlong == 0 && h.nspa == 0) ? 1 : 0;
     ws_expand_kernel<V, NUM><<<unsigned(std::min<int64_t>(ceil_div(nnz, 256), 148 * 32)), 256, 0, s>>>(
         nnz, sw.arow, sw.wmode, sw.S, sw.bstart, static_cast<const V *>(A->vals), B->col_idx,
-        static_cast<const V *>(B->vals), mw.xcol, mw.xval);
+        static_cast<const V *>(B->vals), mw.xcol, mw.xval, all_small);
     msp_status st = last_launch(NUM ? "ws_expand_kernel<numeric>" : "ws_expand_kernel<symbolic>");
     if (st != MSP_OK) return st;
     auto kern = ws_small_kernel<V, NUM>;
@@ -2005,8 +2008,8 @@ msp_status run_rowacc(const msp_csr *A, const msp_csr *B, const SetupWs &sw, con
 {
     const int32_t m = A->nrows;
     if (h.nsmall > 0) {
-        msp_status st = (A->dtype == MSP_F64) ? run_small<double, NUM>(A, B, sw, mw, Crp, Ccol, Cval, s)
-                                              : run_small<float, NUM>(A, B, sw, mw, Crp, Ccol, Cval, s);
+        msp_status st = (A->dtype == MSP_F64) ? run_small<double, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s)
+                                              : run_small<float, NUM>(A, B, sw, mw, h, Crp, Ccol, Cval, s);
         if (st != MSP_OK) return st;
     }
     if (h.nbitmap <= 0) return MSP_OK;
