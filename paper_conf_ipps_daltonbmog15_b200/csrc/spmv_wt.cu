@@ -525,7 +525,10 @@ msp_status launch_wt(const msp_csr *A, const void *x, void *y, void *ws, size_t 
 #endif
     constexpr int NSUB0 = MSP_WT_NSUB > 0 ? MSP_WT_NSUB
                                           : (188 * 1024 / MSP_WT_STAGES) / int((4 + sizeof(V)) * 32 * K);
-    using C = WtCfg<V, K, 11, (NSUB0 < 24 ? NSUB0 : 24), MSP_WT_STAGES>;
+#ifndef MSP_WT_NW
+#define MSP_WT_NW 11  // worker warps (tuning builds)
+#endif
+    using C = WtCfg<V, K, MSP_WT_NW, (NSUB0 < 24 ? NSUB0 : 24), MSP_WT_STAGES>;
     auto kern = spmv_wt_kernel<V, C>;
     int occ = 1;
     static const bool fit = getenv("MSP_SPMV_WT_L1") != nullptr;  // experiment: carveout fitted to the CTA
