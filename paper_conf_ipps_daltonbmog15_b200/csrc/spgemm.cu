@@ -1131,9 +1131,8 @@ struct SetupWs {
                                 //       too wide for the row accumulator (small path off), [8] widest
                                 //       BITMAP span, [9] SMALL rows, [10] BITMAP rows, [11] promoted rows
     int32_t *spanlo, *spanhi;   // [m] output column span of each long row (segmented path, f3)
-    int32_t *spaflag;           // [m] 1 = the row takes the segmented path
-    int64_t *spapos;            // [m + 1]
-    int32_t *sparow;            // [m] rows of the segmented path
+    int32_t *spaflag;           // [m] windows of the row on the segmented path (0: not segmented)
+    int64_t *spapos;            // [m + 1] exclusive scan of spaflag: first window item of each row
     int32_t *bstart;            // [nnzA] B row start of each A nonzero (Brp[Acol[j]])
     uint8_t *wmode;             // [m] warp-row path mode of each short row (WM_*)
     void *scan;
@@ -1161,7 +1160,6 @@ SetupWs carve_setup(const msp_csr *A, void *ws, size_t cap, bool *ok)
     w.spanhi = cv.take<int32_t>(size_t(m > 0 ? m : 1));
     w.spaflag = cv.take<int32_t>(size_t(m > 0 ? m : 1));
     w.spapos = cv.take<int64_t>(size_t(m + 1));
-    w.sparow = cv.take<int32_t>(size_t(m > 0 ? m : 1));
     w.bstart = cv.take<int32_t>(size_t(nnz > 0 ? nnz : 1));
     w.wmode = cv.take<uint8_t>(size_t(m > 0 ? m : 1));
     w.scan_bytes = scan_ws_bytes(std::max<int64_t>(std::max<int64_t>(m, nnz), 1));
