@@ -376,7 +376,10 @@ constexpr int WR_SYM_WARPS = MSP_WR_SYM_WARPS;
 #ifndef WR_EMIT_SERIAL
 #define WR_EMIT_SERIAL 0  // experiment: per-lane serial emission of the column list (C2 symbolic 2.25 -> 3.12 ms: slower)
 #endif           // 64 KB of bitmaps per CTA
-constexpr int WR_UMAX = 512;              // accumulator entries per warp per pass (6 KB with the column list)
+#ifndef MSP_WR_UMAX
+#define MSP_WR_UMAX 512
+#endif
+constexpr int WR_UMAX = MSP_WR_UMAX;      // accumulator entries per warp per pass (6 KB with the column list)
 constexpr int WR_NUM_WARPS = MSP_WR_NUM_WARPS;
 
 __device__ __forceinline__ int warp_excl_sum(int v, int lane, int *total)
@@ -982,7 +985,7 @@ wr_symbolic_kernel(int32_t m, int nw_max, const int32_t *__restrict__ Arp, const
 // rank per 32-bit slot, linear probing) gives each product's rank in one or
 // two shared-memory probes; products accumulate into shared memory in k
 // order.  WR_UMAX columns per pass.
-constexpr int WR_HSLOTS = 2 * WR_UMAX;
+constexpr int WR_HSLOTS = 1024;  // hash slots per warp (load <= 1/2 at WR_UMAX = 512)
 constexpr uint32_t WR_EMPTY = 0xffffffffu;
 constexpr int WR_NUM_SMEM = WR_NUM_WARPS * (WR_UMAX * 8 + WR_HSLOTS * 4);
 
