@@ -43,6 +43,9 @@ namespace {
 #define MSP_ADD_NT 128  // threads per tile: C3 one pass 0.880 -> 0.865 ms, C2 0.410 -> 0.389 ms vs 256 (64-512 swept)
 #endif
 constexpr int ADD_NT = MSP_ADD_NT;
+#ifndef MSP_LB_BACKOFF
+#define MSP_LB_BACKOFF 0  // 1: look-back spin with __nanosleep backoff (C3 0.882 -> 0.872 ms, C2 0.390 -> 0.410 ms: off)
+#endif
 #ifndef MSP_ADD_IPT
 #define MSP_ADD_IPT 14  // measured on B200 (one-walk fill, 53-66 KB smem): C3 A+A^T 1.85 ms at 8, 1.42 at 12,
                         // 1.30 at 14, 1.31 at 16, 1.23 at 20; C2 0.47-0.49 ms at 12-20
@@ -427,9 +430,18 @@ spadd_tile_kernel(int32_t m, const int32_t *__restrict__ Arp, const int32_t *__r
                         const int q = pos - lane;
                         uint64_t sw = AS_PRE;  // virtual prefix 0 before tile 0
                         if (q >= 0) {
-                            do {
+                            sw = *reinterpret_cast<volatile uint64_t *>(&states[q]);
+#if MSP_LB_BACKOFF
+                            // predecessor not published yet: back off (the spin
+                            // took 18 % of the kernel's issued instructions)
+                            for (unsigned ns = 32; (sw & ~AS_VAL) == 0; ns = ns < 256 ? 2 * ns : ns) {
+                                __nanosleep(ns);
                                 sw = *reinterpret_cast<volatile uint64_t *>(&states[q]);
-                            } while ((sw & ~AS_VAL) == 0);  // predecessor not published yet
+                            }
+#else
+                            while ((sw & ~AS_VAL) == 0)  // predecessor not published yet
+                                sw = *reinterpret_cast<volatile uint64_t *>(&states[q]);
+#endif
                         }
                         const unsigned pre = __ballot_sync(0xffffffffu, (sw & AS_PRE) != 0);
                         const int stop = pre ? __ffs(pre) - 1 : 32;  // nearest predecessor with a prefix
