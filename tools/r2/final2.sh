@@ -1,5 +1,5 @@
 set -x
-D=gpurun_out/final4; mkdir -p $D
+D=gpurun_out/final5; mkdir -p $D
 python -c "import __graft_entry__ as g; g.smoke()" > $D/smoke.log 2>&1; echo smoke $?
 timeout 1800 python -m pytest tests -m gpu -q > $D/gputests.log 2>&1; echo tests $?
 timeout 900 python bench.py > $D/bench.log 2>&1; echo bench $?
