@@ -97,11 +97,14 @@ def windowed(seed, mode="random"):
             gen.CSR(kb, n, brp, bcol, gen.matrices.random_values(bcol.size, seed + 1)))
 
 
-@pytest.mark.parametrize("mode", ["random", "int"])
+@pytest.mark.parametrize("mode", ["random", "int", "fp32"])
 def test_windowed_wide_rows(mode):
     """Spans wider than 12,288 columns cut into windows, one CTA each; a
     window's output goes after the row's earlier windows' outputs."""
-    A, B = windowed(8, mode)
+    A, B = windowed(8, "random" if mode == "fp32" else mode)
+    if mode == "fp32":
+        A = A.with_values(A.val.astype(np.float32))
+        B = B.with_values(B.val.astype(np.float32))
     (rp, col, val), info = run(A, B)
     W, sc, _ = oracle.spgemm(A, B)
     spans = [(W.col[W.rp[r + 1] - 1] - W.col[W.rp[r]] + 1) for r in range(A.m)]
